@@ -1,0 +1,425 @@
+#!/usr/bin/env python
+"""Benchmark of libipt's 3-stage in-place transposition on B200 (driver contract).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--workload sweep|c1|c3|c4|c5]
+
+Metric (BASELINE.json): in-place transpose effective GB/s = 2*M*N*elem_bytes / time
+(PAPER.md P:56), whole job (all ranks); also reported as a fraction of the measured HBM
+peak scaled by the stage count S.
+
+Default workload (N = 1): BASELINE.json configs[1], the float32 shape sweep with
+M, N in [1000, 20000].  One step = one in-place transpose of
+every matrix of the sweep (each matrix alternates between M x N and N x M from step to
+step; every matrix is larger than L2, so no flush is needed between steps).  Multi-GPU:
+every rank runs the same per-GPU work on its own GPU (weak scaling, no collective on the
+data path); --workload c5 instead shards 512 matrices across ranks (strong scaling).
+
+Reference arm (--impl reference): the repo's CPU oracle (oracle/, plain single-thread C
+cycle following), timed on the host on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "in-place transpose effective GB/s (2·M·N·bytes/time), % of B200 HBM peak"
+
+SWEEP = [(7200, 18000), (18000, 7200), (16384, 16384), (12800, 15000), (19200, 10000),
+         (9998, 12288), (14803, 8192), (20000, 20000)]
+WORKLOADS = {
+    "sweep": dict(name="configs[1] shape sweep, float32, M,N in [1000,20000]", shapes=SWEEP, eb=4),
+    "c1": dict(name="configs[0] single 1800x7200 float32", shapes=[(1800, 7200)], eb=4),
+    "c3": dict(name="configs[2] skinny 1000000x256 float32", shapes=[(1_000_000, 256)], eb=4),
+    "c4": dict(name="configs[3] large 20000x30000 float64", shapes=[(20000, 30000)], eb=8),
+    "c5": dict(name="configs[4] batch of 512 4096x3000 float32", shapes=[(4096, 3000)], eb=4,
+               batch=512),
+}
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+# ------------------------------------------------------------------------ helpers
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    def __init__(self, index: int):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={index}", f"--query-gpu={q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        rows = []
+        for line in open(self.f.name):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                rows.append((float(parts[1]), float(parts[2]), parts[5:9]))
+            except ValueError:
+                continue
+        os.unlink(self.f.name)
+        if not rows:
+            return None
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for _, _, r in rows for i, v in enumerate(r) if v.lower() == "active"})
+        return {"sm_mhz": statistics.median(r[0] for r in rows),
+                "sm_max_mhz": max(r[1] for r in rows), "reasons": reasons, "samples": len(rows)}
+
+
+def dist_setup():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+# ------------------------------------------------------------ CPU oracle (baseline)
+def oracle_sample(shapes, eb, budget_s=12.0, max_mats=None):
+    """Time the CPU oracle (as it stands) on a bounded sample of the workload."""
+    import numpy as np
+    from inputs import seeded
+    from oracle import oracle
+
+    oracle.build()
+    done_bytes, t_total, used = 0, 0.0, []
+    for (M, N) in shapes:
+        a = seeded.matrix_np(M, N, eb)
+        t0 = time.perf_counter()
+        oracle.transpose_inplace(a, M, N)
+        dt = time.perf_counter() - t0
+        # spot-check the oracle's own result against the definition
+        rnd = np.random.default_rng(0)
+        ks = rnd.integers(0, M * N, 64)
+        i, j = ks // N, ks % N
+        assert np.array_equal(a[j * M + i], seeded.values_np(ks, eb))
+        done_bytes += 2 * M * N * eb
+        t_total += dt
+        used.append(f"{M}x{N}")
+        del a
+        if t_total >= budget_s or (max_mats and len(used) >= max_mats):
+            break
+    return done_bytes, t_total, used
+
+
+def run_reference(args, world, rank):
+    if rank != 0:
+        return 0
+    wl = WORKLOADS[args.workload]
+    shapes = wl["shapes"]
+    # one step = the oracle on one matrix of the workload (bounded: the smallest one)
+    sample = min(shapes, key=lambda s: s[0] * s[1])
+    for _ in range(args.warmup):
+        oracle_sample([sample], wl["eb"], budget_s=0)
+    tot_b, tot_t = 0, 0.0
+    for _ in range(args.steps):
+        b, t, _ = oracle_sample([sample], wl["eb"], budget_s=0)
+        tot_b += b
+        tot_t += t
+    value = tot_b / tot_t / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(1e3 * tot_t / args.steps, 3), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": wl["name"], "sample": f"{sample[0]}x{sample[1]} per step",
+                   "elem_bytes": wl["eb"]},
+        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": f"one {sample[0]}x{sample[1]} matrix per step, single thread C"},
+        "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# -------------------------------------------------------------------------- ours
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="sweep", choices=sorted(WORKLOADS))
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--queues", type=int, default=4)
+    args = ap.parse_args()
+    world, rank, local = dist_setup()
+
+    if args.impl == "reference":
+        return run_reference(args, world, rank)
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ppopp_sunggggh14_b200 as ipt
+    from inputs import seeded
+
+    assert args.warmup >= 3, "timing rules: at least 3 warm-up steps"
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    wl = WORKLOADS[args.workload]
+    eb = wl["eb"]
+    tdt = torch.int32 if eb == 4 else torch.int64
+    stream = torch.cuda.current_stream()
+
+    # ---- matrices resident in HBM, filled on the device by the seeded generator
+    mats = []   # (tensor, M, N, count, t0)
+    if "batch" in wl:
+        M, N = wl["shapes"][0]
+        tot = wl["batch"]
+        lo, hi = tot * rank // world, tot * (rank + 1) // world
+        t = torch.empty((hi - lo) * M * N, dtype=tdt, device=dev)
+        seeded.fill_device_(t, M, N, eb, t0=lo, count=hi - lo)
+        mats.append([t, M, N, hi - lo, lo])
+    else:
+        for (M, N) in wl["shapes"]:
+            t = torch.empty(M * N, dtype=tdt, device=dev)
+            seeded.fill_device_(t, M, N, eb)
+            mats.append([t, M, N, 1, 0])
+    torch.cuda.synchronize()
+    plans = {}
+    for (_, M, N, _, _) in mats:
+        plans[(M, N)] = ipt.plan(M, N, eb, local)
+        plans[(N, M)] = ipt.plan(N, M, eb, local)
+    ws_bytes = max(ipt.workspace_bytes(p, mt[3]) for mt in mats for p in (plans[(mt[1], mt[2])], plans[(mt[2], mt[1])]))
+    ws = torch.empty(max(ws_bytes, 256), dtype=torch.uint8, device=dev)
+    orient = [False] * len(mats)   # False: currently M x N; True: currently N x M
+
+    def one_step(evs=None):
+        for i, (t, M, N, cnt, _) in enumerate(mats):
+            a, b = (N, M) if orient[i] else (M, N)
+            p = plans[(a, b)]
+            if cnt > 1:
+                ipt.transpose_batched_(t, cnt, a, b, plan_=p)
+            else:
+                ipt.transpose_(t, a, b, plan_=p, workspace=ws,
+                               events=evs[i] if evs is not None else None)
+            orient[i] = not orient[i]
+
+    for _ in range(args.warmup):
+        one_step()
+    torch.cuda.synchronize()
+
+    # per-stage events for every matrix and every step (created by one record each)
+    evs = [[[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in mats]
+           for _ in range(args.steps)]
+    for s in evs:
+        for m in s:
+            for e in m:
+                e.record()
+    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks = ClockSampler(local)
+    launches0 = ipt.kernel_launch_count()
+    orient_before = list(orient)
+    t_start.record()
+    for s in range(args.steps):
+        one_step(evs[s] if "batch" not in wl else None)
+    t_end.record()
+    torch.cuda.synchronize()
+    launches = ipt.kernel_launch_count() - launches0
+    clk = clocks.stop()
+    elapsed_ms = t_start.elapsed_time(t_end)
+    tmax = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.barrier()
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+    elapsed_ms = float(tmax.item())
+
+    # ---- throughput
+    bytes_per_step_rank = sum(2 * M * N * eb * cnt for (_, M, N, cnt, _) in mats)
+    total_units = bytes_per_step_rank * args.steps * (world if "batch" not in wl else 1)
+    if "batch" in wl:
+        M, N = wl["shapes"][0]
+        total_units = 2 * M * N * eb * wl["batch"] * args.steps
+    value_gbs = total_units / (elapsed_ms / 1e3) / 1e9
+    peak, peak_src = load_peaks()
+
+    # ---- per-stage (per-kernel) live timing -> roofline of the dominant kernel
+    kern_t = {"cycle_global": 0.0, "tile_onchip": 0.0}
+    kern_bytes = {"cycle_global": 0, "tile_onchip": 0}
+    kern_n = {"cycle_global": 0, "tile_onchip": 0}
+    stage_scaled = None
+    if "batch" not in wl:
+        orient_sim = list(orient_before)
+        S_bytes = 0
+        for s in range(args.steps):
+            for i, (t, M, N, cnt, _) in enumerate(mats):
+                a, b = (N, M) if orient_sim[i] else (M, N)
+                p = plans[(a, b)]
+                for st in range(3):
+                    v = ipt.VARIANTS[p.variant[st]]
+                    if v == "identity":
+                        continue
+                    dt = evs[s][i][st].elapsed_time(evs[s][i][st + 1])
+                    kern_t[v] += dt
+                    kern_bytes[v] += 2 * a * b * eb
+                    kern_n[v] += 1
+                    S_bytes += 2 * a * b * eb
+                orient_sim[i] = not orient_sim[i]
+        stage_scaled = (S_bytes / (elapsed_ms / 1e3) / 1e9) / peak
+    dom = max(kern_t, key=lambda k: kern_t[k]) if any(kern_t.values()) else None
+    roofline = None
+    if dom:
+        achieved = kern_bytes[dom] / (kern_t[dom] / 1e3) / 1e9
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", "traffic.json")
+        if os.path.exists(tp):
+            try:
+                traffic = json.load(open(tp)).get(args.workload, {}).get(dom)
+            except Exception:
+                traffic = None
+        roofline = {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 1), "peak": peak,
+                    "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
+                    "peak_source": peak_src, "launches": kern_n[dom],
+                    "avg_launch_ms": round(kern_t[dom] / max(1, kern_n[dom]), 4),
+                    "share_of_step": round(kern_t[dom] / elapsed_ms, 4),
+                    "per_kernel_ms": {k: round(v, 3) for k, v in kern_t.items()}}
+
+    # ---- verification of the final state (sampled, definition-based on device)
+    ok = True
+    for i, (t, M, N, cnt, t0) in enumerate(mats):
+        transposed = orient[i]
+        a, b = (M, N) if not transposed else (N, M)   # current shape a x b
+        n = M * N
+        g = torch.Generator(device="cpu").manual_seed(i)
+        for k in range(min(cnt, 3)):
+            pos = torch.randint(0, n, (4096,), generator=g).to(dev)
+            seg = t[k * n:(k + 1) * n] if cnt > 1 else t
+            if transposed:   # position p = j*M + i holds v(i*N + j)
+                src = (pos % M) * N + pos // M
+            else:
+                src = pos
+            exp = seeded.values_torch_sample(src + (t0 + k) * n, eb)
+            if not torch.equal(seg[pos], exp.to(seg.dtype)):
+                ok = False
+    del ws
+    # ---- e2e through the public host API (H2D + 3 stages + D2H, Sec. 6)
+    e2e = None
+    if not args.no_e2e and "batch" not in wl:
+        hosts = []
+        for (_, M, N, _, _) in mats:
+            hosts.append([torch.empty(M * N, dtype=tdt, pin_memory=True), M, N])
+        for (h, M, N) in hosts:
+            tmp = torch.empty(M * N, dtype=tdt, device=dev)
+            seeded.fill_device_(tmp, M, N, eb)
+            h.copy_(tmp)
+            del tmp
+        for t_ in mats:
+            t_[0] = None
+        mats.clear()
+        torch.cuda.empty_cache()
+        horient = [False] * len(hosts)
+
+        def e2e_step():
+            for i, (h, M, N) in enumerate(hosts):
+                a, b = (N, M) if horient[i] else (M, N)
+                ipt.transpose_host_(h, a, b, queues=args.queues)
+                horient[i] = not horient[i]
+
+        e2e_step()   # warm-up (allocates the device staging buffer)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        w0 = time.perf_counter()
+        e0.record()
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        e1.record()
+        torch.cuda.synchronize()
+        wall = time.perf_counter() - w0
+        ems = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(ems, op=dist.ReduceOp.MAX)
+        hb = sum(M * N * eb for (_, M, N) in hosts)
+        e2e = {"value": round(hb * 2 * args.e2e_steps * world / (float(ems.item()) / 1e3) / 1e9, 3),
+               "unit": "GB/s", "h2d_bytes_per_step": hb, "d2h_bytes_per_step": hb,
+               "steps": args.e2e_steps, "queues": args.queues, "wall_s": round(wall, 3),
+               "api": "ipt_transpose_host (pinned host buffers)"}
+        # verify one host result
+        (h, M, N) = hosts[0]
+        idx = torch.randint(0, M * N, (2048,))
+        src = (idx % M) * N + idx // M if horient[0] else idx
+        if not torch.equal(h[idx], seeded.values_torch_sample(src, eb).to(h.dtype)):
+            ok = False
+
+    # ---- CPU oracle baseline (rank 0, N = 1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        shapes = [(M, N) for (M, N) in wl["shapes"]]
+        b, t, used = oracle_sample(shapes, eb, budget_s=12.0)
+        cpu = {"value": round(b / t / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+               "sample": f"{'+'.join(used)} ({eb}-byte elements), single-thread C cycle following",
+               "host_cpus": os.cpu_count()}
+
+    if rank == 0:
+        plans_cfg = {f"{M}x{N}": {"m": p.m, "n": p.n, "S": p.n_stages,
+                                  "variant": [ipt.VARIANTS[v] for v in p.variant]}
+                     for (M, N), p in plans.items()}
+        line = {
+            "metric": METRIC, "value": round(value_gbs, 2), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(elapsed_ms / args.steps, 4), "higher_is_better": True,
+            "scaling": "weak" if "batch" not in wl else "strong", "vs_baseline": None,
+            "dtype": "u32" if eb == 4 else "u64", "data": "synthetic",
+            "config": {"workload": wl["name"],
+                       "shapes": [f"{M}x{N}" for (M, N) in wl["shapes"]],
+                       "elem_bytes": eb, "batch": wl.get("batch", 1),
+                       "plans": plans_cfg,
+                       "l2": "no flush: every matrix exceeds the 126 MB L2" if args.workload in ("sweep", "c3", "c4", "c5") else "L2-resident (52 MB)",
+                       "parallelism": f"replicas x{world}" if "batch" not in wl else f"batch shards x{world}"},
+            "hbm_frac_stage_scaled": round(stage_scaled, 4) if stage_scaled else None,
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
+            "clocks": clk, "verified": ok,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0 if ok else 1
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,184 @@
+/*
+ * ipt.h -- C ABI of libipt, a B200-native (sm_100a) in-place matrix transposition
+ * library following Sung, Gomez-Luna, Gonzalez-Linares, Guil, Hwu, "In-Place
+ * Transposition of Rectangular Matrices on Accelerators", PPoPP'14.
+ *
+ * Citations "P:<line>" refer to the paper text line, with the section /
+ * equation it falls in.  SURVEY.md 8(b) is the contract this header implements.
+ *
+ * THE OPERATION (Sec. 3).  A is an M x N row-major array of elements of
+ * `elem_bytes` bytes; after ipt_transpose the same storage holds A^T, the N x M
+ * row-major array with A^T(j, i) = A(i, j); i.e. the byte content of offset
+ * k = i*N + j moves to k' = j*M + i (Eq. (1)).  Elements are moved as raw
+ * bytes (no floating-point operation; NaN payloads survive).
+ *
+ * THE METHOD (Sec. 4.2).  With M = M'*m and N = N'*n the transpose is
+ * the composition of three elementary tiled transpositions ("stages"):
+ *   stage 1  100!  : M x N' x n        -> N' x M x n
+ *   stage 2  0010! : N' x M' x m x n   -> N' x M' x n x m
+ *   stage 3  0100! : N' x M' x n x m   -> N' x n x M' x m
+ * Every elementary transposition swaps two adjacent dimensions of a row-major array,
+ * so all of them are instances of one operation:
+ *   P(batch, A, B, s) : batch x [A x B x s]  ->  batch x [B x A x s]
+ * ("super-elements" of s contiguous elements are shifted as a whole).
+ *
+ * CONVENTIONS (the paper is silent):
+ *   - Ownership: the caller owns every data pointer; libipt never allocates or frees it.
+ *   - Device pointers ("d_"): CUDA device memory of the current device.  Host pointers
+ *     ("h_"): host memory (pinned or pageable).
+ *   - Asynchrony: every device call is stream-ordered on `stream` (a cudaStream_t; NULL =
+ *     legacy default stream) and returns after enqueueing.  Host calls (ipt_*_host)
+ *     return after the result is back in host memory.
+ *   - Validation: all arguments are checked BEFORE any launch; an error return other
+ *     than IPT_ERR_CUDA means nothing was enqueued and the data is untouched.
+ *   - Errors after launch return IPT_ERR_CUDA; the data is then undefined (an in-place
+ *     permutation is not resumable: the flag bitmap is the only progress record).
+ *   - elem_bytes in {1, 2, 4, 8, 16}; the data pointer must be aligned to elem_bytes.
+ *     16-byte vector paths are selected automatically when alignment permits.
+ *   - Workspace: cycle-following stages need one flag bit per moved unit plus a work
+ *     counter ("only one bit per super-element is needed").  Pass a device
+ *     buffer of ipt_workspace_bytes() bytes, or NULL to use an internal per-(device,
+ *     stream) cache.  libipt zeroes the flags itself before every stage.
+ *   - Thread safety: concurrent calls on distinct buffers with distinct workspaces (or
+ *     distinct streams when using the internal cache) are safe.
+ *   - M == 1 or N == 1 (and empty batches) are successful no-ops.
+ */
+#ifndef IPT_H
+#define IPT_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    IPT_OK = 0,
+    IPT_ERR_INVALID_ARG = 1,      /* a size < 0 / < 1, NULL pointer, overflow          */
+    IPT_ERR_UNSUPPORTED_ELEM = 2, /* elem_bytes not in {1,2,4,8,16}                    */
+    IPT_ERR_MISALIGNED = 3,       /* data pointer / stride not aligned to elem_bytes   */
+    IPT_ERR_NO_MEMORY = 4,        /* workspace too small / internal allocation failed  */
+    IPT_ERR_CUDA = 5,             /* a CUDA call failed (data undefined if after launch) */
+    IPT_ERR_NO_DEVICE = 6         /* device query failed (no CUDA device)              */
+} ipt_status;
+
+/* How one stage is executed. */
+typedef enum {
+    IPT_VAR_IDENTITY = 0,      /* stage elided: a swapped dimension is 1 */
+    IPT_VAR_TILE_ONCHIP = 1,   /* whole tile staged in shared memory (BS, Fig. 1) */
+    IPT_VAR_CYCLE_ONCHIP = 2,  /* PTTWAC inside a tile, flag bits in shared memory */
+    IPT_VAR_CYCLE_GLOBAL = 3   /* PTTWAC over super-elements, flag bits in global memory */
+} ipt_variant;
+
+/* A plan for the 3-stage transposition of one M x N matrix (Sec. 4.2 + Sec. 7.4). */
+typedef struct {
+    int64_t M, N;          /* matrix shape                                     */
+    int64_t m, n;          /* tile sizes: M = Mp*m, N = Np*n            */
+    int64_t Mp, Np;        /* M' and N'                                         */
+    int32_t elem_bytes;
+    int32_t n_stages;      /* number of non-identity stages (S in the roofline) */
+    int32_t variant[3];    /* ipt_variant of stage 1, 2, 3                      */
+    int32_t reserved;
+    int64_t flag_bits[3];  /* flag bits used by each stage for ONE matrix       */
+    uint64_t workspace_bytes; /* device workspace for ONE matrix (max over stages) */
+} ipt_plan_t;
+
+/* ---------------------------------------------------------------- planning (host) */
+
+/* Tile-size planner (Sec. 7.4): factors M and N and picks (m, n) and a
+ * variant per stage from a cost model of the B200 kernels.  Host-only, deterministic
+ * for a given (M, N, elem_bytes, device properties).  device < 0 plans for a nominal
+ * B200 (148 SMs, 227 KB shared memory per block) without touching the GPU. */
+ipt_status ipt_plan(int64_t M, int64_t N, int elem_bytes, int device, ipt_plan_t *out);
+
+/* Same with forced tile sizes m | M and n | N (IPT_ERR_INVALID_ARG otherwise). */
+ipt_status ipt_plan_with_tiles(int64_t M, int64_t N, int64_t m, int64_t n, int elem_bytes,
+                               int device, ipt_plan_t *out);
+
+/* Device workspace bytes for executing `plan` on a batch of `batch` matrices. */
+size_t ipt_workspace_bytes(const ipt_plan_t *plan, int64_t batch);
+
+/* ------------------------------------------------------------ full transposition */
+
+/* A (M x N, row-major, at d_ptr) -> A^T (N x M) in the same storage. */
+ipt_status ipt_transpose(void *d_ptr, int64_t M, int64_t N, int elem_bytes, void *stream);
+
+/* Executes a given plan.  d_workspace may be NULL (internal cache); otherwise it must
+ * hold ipt_workspace_bytes(plan, 1) bytes (ws_bytes). */
+ipt_status ipt_transpose_plan(void *d_ptr, const ipt_plan_t *plan, void *d_workspace,
+                              size_t ws_bytes, void *stream);
+
+/* As ipt_transpose_plan, and records `events` (cudaEvent_t[4], each may be NULL) on the
+ * stream: events[0] before stage 1, events[i] right after stage i (identity stages
+ * record at the same point).  Used to time each stage live. */
+ipt_status ipt_transpose_plan_events(void *d_ptr, const ipt_plan_t *plan, void *d_workspace,
+                                     size_t ws_bytes, void *stream, void *const *events);
+
+/* `count` independent M x N matrices, matrix t at d_base + t*stride_bytes
+ * (stride_bytes >= M*N*elem_bytes, multiple of elem_bytes).  The batch is folded into
+ * each stage (the instances are independent), so each stage is one launch. */
+ipt_status ipt_transpose_batched(void *d_base, int64_t count, int64_t stride_bytes,
+                                 int64_t M, int64_t N, int elem_bytes, void *stream);
+
+ipt_status ipt_transpose_batched_plan(void *d_base, int64_t count, int64_t stride_bytes,
+                                      const ipt_plan_t *plan, void *d_workspace,
+                                      size_t ws_bytes, void *stream);
+
+/* ----------------------------------------------- host-delegated transposition (Sec. 6) */
+
+/* In-place transposition of a HOST array executed on the GPU (Fig. 4/5):
+ * host->device copy, stage 1 on `stream`, then stages 2-3 and the device->host copy split
+ * into `queues` groups of output panels on separate streams so that transfers overlap the
+ * remaining stages (Fig. 5b; queues = 1 is the synchronous scheme of Fig. 5a).  h_ptr is
+ * read and overwritten with A^T (N x M); pinned host memory is required for overlap.
+ * d_buffer (device, may be NULL = internal cache) must hold at least M*N*elem_bytes plus
+ * the flag workspace (IPT_ERR_NO_MEMORY otherwise).  Returns after the result is in
+ * host memory. */
+ipt_status ipt_transpose_host(void *h_ptr, int64_t M, int64_t N, int elem_bytes, int queues,
+                              void *d_buffer, size_t d_buffer_bytes, void *stream);
+
+/* ------------------------------------------------ elementary transpositions */
+
+/* Device workspace bytes for P(batch, A, B, s) with elem_bytes elements. */
+size_t ipt_stage_workspace_bytes(int64_t batch, int64_t A, int64_t B, int64_t s,
+                                 int elem_bytes);
+
+/* 100! (SoA -> ASTA, Sec. 5.2): batch x [A x B x s] -> batch x [B x A x s] by
+ * cycle following of s-element super-elements with one global flag bit each. */
+ipt_status ipt_100(void *d_ptr, int64_t batch, int64_t A, int64_t B, int64_t s,
+                   int elem_bytes, void *d_workspace, size_t ws_bytes, void *stream);
+
+/* 010! (AoS -> ASTA, Sec. 5.1): batch x [A x B] -> batch x [B x A] (tile-local
+ * transposes; on-chip when a tile fits shared memory, else cycle following). */
+ipt_status ipt_010(void *d_ptr, int64_t batch, int64_t A, int64_t B, int elem_bytes,
+                   void *d_workspace, size_t ws_bytes, void *stream);
+
+/* 0010! on a 4-D array d0 x d1 x d2 x d3 -> d0 x d1 x d3 x d2 (= ipt_010(d0*d1, d2, d3)). */
+ipt_status ipt_0010(void *d_ptr, int64_t d0, int64_t d1, int64_t d2, int64_t d3,
+                    int elem_bytes, void *d_workspace, size_t ws_bytes, void *stream);
+
+/* 0100! on a 4-D array d0 x d1 x d2 x d3 -> d0 x d2 x d1 x d3 (= ipt_100(d0, d1, d2, d3)). */
+ipt_status ipt_0100(void *d_ptr, int64_t d0, int64_t d1, int64_t d2, int64_t d3,
+                    int elem_bytes, void *d_workspace, size_t ws_bytes, void *stream);
+
+/* 1000! on a 4-D array d0 x d1 x d2 x d3 -> d1 x d0 x d2 x d3 (= ipt_100(1, d0, d1, d2*d3));
+ * the third stage of the 4-stage Gustavson/Karlsson scheme. */
+ipt_status ipt_1000(void *d_ptr, int64_t d0, int64_t d1, int64_t d2, int64_t d3,
+                    int elem_bytes, void *d_workspace, size_t ws_bytes, void *stream);
+
+/* ------------------------------------------------------------------- diagnostics */
+
+const char *ipt_status_string(ipt_status s);
+
+/* Number of libipt kernels launched by this process so far (all devices). */
+uint64_t ipt_kernel_launch_count(void);
+
+/* Library version string. */
+const char *ipt_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* IPT_H */

@@ -1,0 +1,534 @@
+// ipt_api.cpp -- the C ABI of libipt (include/ipt.h): argument validation, plan
+// execution (stage sequencing on one stream), workspace management, diagnostics.
+//
+// Stage sequence (Sec. 4.2) for `count` matrices at base + t*stride:
+//   stage 1  100!  P(count, M, N', n)          -> cycle_global  (or identity)
+//   stage 2  0010! P(count*N'*M', m, n, 1)     -> tile_onchip / cycle_global (or identity)
+//   stage 3  0100! P(count*N', M', n, m)       -> cycle_global  (or identity)
+// The batch is folded into every stage (the instances are independent), so each
+// stage is a single launch regardless of `count`.
+#include "ipt_internal.h"
+
+#include <algorithm>
+#include <atomic>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <vector>
+
+namespace ipt {
+
+ipt_status plan_search(int64_t M, int64_t N, int eb, int device, ipt_plan_t *out);
+void fill_plan(int64_t M, int64_t N, int64_t m, int64_t n, int eb, int device, ipt_plan_t *out);
+
+static std::atomic<uint64_t> g_launches{0};
+void note_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+
+long env_int(const char *name, long dflt) {
+    const char *v = std::getenv(name);
+    if (!v || !*v) return dflt;
+    char *end = nullptr;
+    long x = std::strtol(v, &end, 10);
+    return (end && *end == 0) ? x : dflt;
+}
+
+FastDiv make_fastdiv(uint64_t d) {
+    FastDiv f{};
+    if (d == 0) d = 1;
+    f.d = d;
+    uint32_t l = 0;
+    if (d > 1) l = 64 - (uint32_t)__builtin_clzll(d - 1);   // ceil(log2 d)
+    unsigned __int128 two_l = (unsigned __int128)1 << l;
+    unsigned __int128 m = ((two_l - d) << 64) / d + 1;
+    f.m = (uint64_t)m;
+    f.s1 = l ? 1 : 0;
+    f.s2 = l ? l - 1 : 0;
+    return f;
+}
+
+DevProps dev_props(int device) {
+    static std::mutex mu;
+    static std::map<int, DevProps> cache;
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = cache.find(device);
+    if (it != cache.end()) return it->second;
+    DevProps p{};
+    // nominal B200 (sm_100a) values, used when planning without a device (device < 0)
+    p.sms = 148;
+    p.smem_optin = 232448;
+    p.smem_per_sm = 233472;
+    p.max_threads_sm = 2048;
+    p.l2_bytes = 126 * 1024 * 1024;
+    p.valid = device < 0;
+    if (device >= 0) {
+        int v = 0;
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, device) == cudaSuccess) {
+            p.sms = v;
+            p.valid = true;
+            cudaDeviceGetAttribute(&p.smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
+            cudaDeviceGetAttribute(&p.smem_per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, device);
+            cudaDeviceGetAttribute(&p.max_threads_sm, cudaDevAttrMaxThreadsPerMultiProcessor, device);
+            cudaDeviceGetAttribute(&p.l2_bytes, cudaDevAttrL2CacheSize, device);
+        } else {
+            cudaGetLastError();
+        }
+    }
+    cache[device] = p;
+    return p;
+}
+
+}  // namespace ipt
+
+using namespace ipt;
+
+namespace {
+
+bool elem_ok(int eb) { return eb == 1 || eb == 2 || eb == 4 || eb == 8 || eb == 16; }
+
+bool mul_ok(int64_t a, int64_t b, int64_t *out) {
+    if (a < 0 || b < 0) return false;
+    if (a == 0 || b == 0) { *out = 0; return true; }
+    if (a > INT64_MAX / b) return false;
+    *out = a * b;
+    return true;
+}
+
+ipt_status check_shape(int64_t M, int64_t N, int eb, int64_t *bytes) {
+    if (!elem_ok(eb)) return IPT_ERR_UNSUPPORTED_ELEM;
+    if (M < 1 || N < 1) return IPT_ERR_INVALID_ARG;
+    int64_t mn = 0, b = 0;
+    if (!mul_ok(M, N, &mn) || !mul_ok(mn, eb, &b)) return IPT_ERR_INVALID_ARG;
+    if (bytes) *bytes = b;
+    return IPT_OK;
+}
+
+int current_device() {
+    int d = 0;
+    if (cudaGetDevice(&d) != cudaSuccess) {
+        cudaGetLastError();
+        return -1;
+    }
+    return d;
+}
+
+// Internal workspace cache, one buffer per (device, stream).
+struct WsCache {
+    std::mutex mu;
+    std::map<std::pair<int, void *>, std::pair<void *, size_t>> bufs;
+};
+WsCache &ws_cache() {
+    static WsCache *c = new WsCache();   // leaked on purpose: outlives CUDA teardown
+    return *c;
+}
+
+ipt_status get_ws(int device, void *stream, size_t need, void **out) {
+    if (need == 0) { *out = nullptr; return IPT_OK; }
+    WsCache &c = ws_cache();
+    std::lock_guard<std::mutex> lk(c.mu);
+    auto key = std::make_pair(device, stream);
+    auto it = c.bufs.find(key);
+    if (it != c.bufs.end() && it->second.second >= need) {
+        *out = it->second.first;
+        return IPT_OK;
+    }
+    if (it != c.bufs.end()) {
+        // previous work on this stream may still use the old buffer
+        cudaStreamSynchronize((cudaStream_t)stream);
+        cudaFree(it->second.first);
+        c.bufs.erase(it);
+    }
+    size_t sz = need < (1u << 20) ? (1u << 20) : need + need / 4;
+    void *p = nullptr;
+    if (cudaMalloc(&p, sz) != cudaSuccess) {
+        cudaGetLastError();
+        return IPT_ERR_NO_MEMORY;
+    }
+    c.bufs[key] = std::make_pair(p, sz);
+    *out = p;
+    return IPT_OK;
+}
+
+ipt_status cuda_status(cudaError_t e) {
+    if (e == cudaSuccess) return IPT_OK;
+    cudaGetLastError();
+    return IPT_ERR_CUDA;
+}
+
+void rec(void *const *events, int i, cudaStream_t st) {
+    if (events && events[i]) cudaEventRecord((cudaEvent_t)events[i], st);
+}
+
+// Stage descriptors of a plan applied to `count` matrices.
+void plan_stages(const ipt_plan_t *p, char *base, int64_t count, int64_t stride, StageDesc st[3]) {
+    for (int i = 0; i < 3; ++i) {
+        st[i] = StageDesc{};
+        st[i].base = base;
+        st[i].outer = count;
+        st[i].ostride = stride;
+        st[i].eb = p->elem_bytes;
+    }
+    st[0].inner = 1;            st[0].A = p->M;  st[0].B = p->Np; st[0].s = p->n;
+    st[1].inner = p->Np * p->Mp; st[1].A = p->m;  st[1].B = p->n;  st[1].s = 1;
+    st[2].inner = p->Np;        st[2].A = p->Mp; st[2].B = p->n;  st[2].s = p->m;
+}
+
+ipt_status validate_plan(const ipt_plan_t *p) {
+    if (!p) return IPT_ERR_INVALID_ARG;
+    ipt_status s = check_shape(p->M, p->N, p->elem_bytes, nullptr);
+    if (s) return s;
+    if (p->m < 1 || p->n < 1 || p->M % p->m || p->N % p->n || p->Mp != p->M / p->m ||
+        p->Np != p->N / p->n)
+        return IPT_ERR_INVALID_ARG;
+    for (int i = 0; i < 3; ++i)
+        if (p->variant[i] < IPT_VAR_IDENTITY || p->variant[i] > IPT_VAR_CYCLE_GLOBAL)
+            return IPT_ERR_INVALID_ARG;
+    return IPT_OK;
+}
+
+size_t batched_ws(const ipt_plan_t *p, int64_t count) {
+    StageDesc st[3];
+    plan_stages(p, nullptr, count, p->M * p->N * p->elem_bytes, st);
+    size_t ws = 0;
+    for (int i = 0; i < 3; ++i)
+        if (p->variant[i] == IPT_VAR_CYCLE_GLOBAL) ws = std::max(ws, cycle_ws_bytes(st[i]));
+    return ws;
+}
+
+ipt_status run_plan(char *base, int64_t count, int64_t stride, const ipt_plan_t *p, void *ws,
+                    size_t ws_bytes, cudaStream_t st, void *const *events) {
+    const int device = current_device();
+    if (device < 0) return IPT_ERR_NO_DEVICE;
+    const size_t need = batched_ws(p, count);
+    if (ws == nullptr) {
+        ipt_status s = get_ws(device, (void *)st, need, &ws);
+        if (s) return s;
+    } else if (ws_bytes < need) {
+        return IPT_ERR_NO_MEMORY;
+    }
+    StageDesc sd[3];
+    plan_stages(p, base, count, stride, sd);
+    rec(events, 0, st);
+    for (int i = 0; i < 3; ++i) {
+        cudaError_t e = cudaSuccess;
+        switch (p->variant[i]) {
+            case IPT_VAR_IDENTITY: break;
+            case IPT_VAR_TILE_ONCHIP: e = launch_tile_onchip(sd[i], st, device); break;
+            case IPT_VAR_CYCLE_ONCHIP:   // not built yet: global-flag cycle following
+            case IPT_VAR_CYCLE_GLOBAL: e = launch_cycle_global(sd[i], ws, st, device); break;
+        }
+        if (e != cudaSuccess) return cuda_status(e);
+        rec(events, i + 1, st);
+    }
+    return IPT_OK;
+}
+
+ipt_status check_ptr(const void *p, int eb) {
+    if (!p) return IPT_ERR_INVALID_ARG;
+    if (((uintptr_t)p) % (uintptr_t)eb) return IPT_ERR_MISALIGNED;
+    return IPT_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+ipt_status ipt_plan(int64_t M, int64_t N, int elem_bytes, int device, ipt_plan_t *out) {
+    if (!out) return IPT_ERR_INVALID_ARG;
+    ipt_status s = check_shape(M, N, elem_bytes, nullptr);
+    if (s) return s;
+    return plan_search(M, N, elem_bytes, device, out);
+}
+
+ipt_status ipt_plan_with_tiles(int64_t M, int64_t N, int64_t m, int64_t n, int elem_bytes,
+                               int device, ipt_plan_t *out) {
+    if (!out) return IPT_ERR_INVALID_ARG;
+    ipt_status s = check_shape(M, N, elem_bytes, nullptr);
+    if (s) return s;
+    if (m < 1 || n < 1 || M % m || N % n) return IPT_ERR_INVALID_ARG;
+    fill_plan(M, N, m, n, elem_bytes, device, out);
+    return IPT_OK;
+}
+
+size_t ipt_workspace_bytes(const ipt_plan_t *plan, int64_t batch) {
+    if (validate_plan(plan) || batch < 0) return 0;
+    return batched_ws(plan, batch);
+}
+
+ipt_status ipt_transpose_plan_events(void *d_ptr, const ipt_plan_t *plan, void *d_workspace,
+                                     size_t ws_bytes, void *stream, void *const *events) {
+    ipt_status s = validate_plan(plan);
+    if (s) return s;
+    if ((s = check_ptr(d_ptr, plan->elem_bytes))) return s;
+    return run_plan((char *)d_ptr, 1, plan->M * plan->N * plan->elem_bytes, plan, d_workspace,
+                    ws_bytes, (cudaStream_t)stream, events);
+}
+
+ipt_status ipt_transpose_plan(void *d_ptr, const ipt_plan_t *plan, void *d_workspace,
+                              size_t ws_bytes, void *stream) {
+    return ipt_transpose_plan_events(d_ptr, plan, d_workspace, ws_bytes, stream, nullptr);
+}
+
+ipt_status ipt_transpose(void *d_ptr, int64_t M, int64_t N, int elem_bytes, void *stream) {
+    ipt_status s = check_shape(M, N, elem_bytes, nullptr);
+    if (s) return s;
+    if ((s = check_ptr(d_ptr, elem_bytes))) return s;
+    if (M == 1 || N == 1) return IPT_OK;
+    const int device = current_device();
+    if (device < 0) return IPT_ERR_NO_DEVICE;
+    ipt_plan_t p;
+    if ((s = ipt_plan(M, N, elem_bytes, device, &p))) return s;
+    return run_plan((char *)d_ptr, 1, M * N * elem_bytes, &p, nullptr, 0, (cudaStream_t)stream,
+                    nullptr);
+}
+
+ipt_status ipt_transpose_batched_plan(void *d_base, int64_t count, int64_t stride_bytes,
+                                      const ipt_plan_t *plan, void *d_workspace,
+                                      size_t ws_bytes, void *stream) {
+    ipt_status s = validate_plan(plan);
+    if (s) return s;
+    if (count < 0) return IPT_ERR_INVALID_ARG;
+    if (count == 0) return IPT_OK;
+    if ((s = check_ptr(d_base, plan->elem_bytes))) return s;
+    const int64_t mat = plan->M * plan->N * plan->elem_bytes;
+    if (count > 1 && (stride_bytes < mat || stride_bytes % plan->elem_bytes)) return IPT_ERR_INVALID_ARG;
+    if (count == 1) stride_bytes = mat;
+    int64_t tot = 0;
+    if (!mul_ok(count - 1, stride_bytes, &tot) || tot > INT64_MAX - mat) return IPT_ERR_INVALID_ARG;
+    return run_plan((char *)d_base, count, stride_bytes, plan, d_workspace, ws_bytes,
+                    (cudaStream_t)stream, nullptr);
+}
+
+ipt_status ipt_transpose_batched(void *d_base, int64_t count, int64_t stride_bytes, int64_t M,
+                                 int64_t N, int elem_bytes, void *stream) {
+    ipt_status s = check_shape(M, N, elem_bytes, nullptr);
+    if (s) return s;
+    if (count < 0) return IPT_ERR_INVALID_ARG;
+    if (count == 0 || M == 1 || N == 1) return IPT_OK;
+    if ((s = check_ptr(d_base, elem_bytes))) return s;
+    const int64_t mat = M * N * elem_bytes;
+    if (count > 1 && (stride_bytes < mat || stride_bytes % elem_bytes)) return IPT_ERR_INVALID_ARG;
+    const int device = current_device();
+    if (device < 0) return IPT_ERR_NO_DEVICE;
+    ipt_plan_t p;
+    if ((s = ipt_plan(M, N, elem_bytes, device, &p))) return s;
+    return ipt_transpose_batched_plan(d_base, count, stride_bytes, &p, nullptr, 0, stream);
+}
+
+// ----------------------------------------------------------- elementary transpositions
+static ipt_status check_stage(void *d, int64_t batch, int64_t A, int64_t B, int64_t s, int eb) {
+    if (!elem_ok(eb)) return IPT_ERR_UNSUPPORTED_ELEM;
+    if (batch < 0 || A < 1 || B < 1 || s < 1) return IPT_ERR_INVALID_ARG;
+    int64_t x = 0;
+    if (!mul_ok(batch, A, &x) || !mul_ok(x, B, &x) || !mul_ok(x, s, &x) || !mul_ok(x, eb, &x))
+        return IPT_ERR_INVALID_ARG;
+    if (batch == 0 || A == 1 || B == 1) return IPT_OK;
+    return check_ptr(d, eb);
+}
+
+static StageDesc stage_desc(void *d, int64_t batch, int64_t A, int64_t B, int64_t s, int eb) {
+    StageDesc sd{};
+    sd.base = (char *)d;
+    sd.outer = batch;
+    sd.inner = 1;
+    sd.ostride = A * B * s * eb;
+    sd.A = A; sd.B = B; sd.s = s; sd.eb = eb;
+    return sd;
+}
+
+size_t ipt_stage_workspace_bytes(int64_t batch, int64_t A, int64_t B, int64_t s, int elem_bytes) {
+    if (check_stage((void *)16, batch, A, B, s, elem_bytes) != IPT_OK) return 0;
+    if (batch == 0 || A == 1 || B == 1) return 0;
+    return cycle_ws_bytes(stage_desc(nullptr, batch, A, B, s, elem_bytes));
+}
+
+static ipt_status run_cycle(void *d, int64_t batch, int64_t A, int64_t B, int64_t s, int eb,
+                            void *ws, size_t ws_bytes, void *stream) {
+    ipt_status st = check_stage(d, batch, A, B, s, eb);
+    if (st) return st;
+    if (batch == 0 || A == 1 || B == 1) return IPT_OK;
+    const int device = current_device();
+    if (device < 0) return IPT_ERR_NO_DEVICE;
+    StageDesc sd = stage_desc(d, batch, A, B, s, eb);
+    const size_t need = cycle_ws_bytes(sd);
+    if (!ws) {
+        if ((st = get_ws(device, stream, need, &ws))) return st;
+    } else if (ws_bytes < need) {
+        return IPT_ERR_NO_MEMORY;
+    }
+    return cuda_status(launch_cycle_global(sd, ws, (cudaStream_t)stream, device));
+}
+
+ipt_status ipt_100(void *d_ptr, int64_t batch, int64_t A, int64_t B, int64_t s, int elem_bytes,
+                   void *d_workspace, size_t ws_bytes, void *stream) {
+    return run_cycle(d_ptr, batch, A, B, s, elem_bytes, d_workspace, ws_bytes, stream);
+}
+
+ipt_status ipt_010(void *d_ptr, int64_t batch, int64_t A, int64_t B, int elem_bytes,
+                   void *d_workspace, size_t ws_bytes, void *stream) {
+    ipt_status st = check_stage(d_ptr, batch, A, B, 1, elem_bytes);
+    if (st) return st;
+    if (batch == 0 || A == 1 || B == 1) return IPT_OK;
+    const int device = current_device();
+    if (device < 0) return IPT_ERR_NO_DEVICE;
+    if (tile_onchip_fits(A, B, elem_bytes, device)) {
+        StageDesc sd = stage_desc(d_ptr, batch, A, B, 1, elem_bytes);
+        return cuda_status(launch_tile_onchip(sd, (cudaStream_t)stream, device));
+    }
+    return run_cycle(d_ptr, batch, A, B, 1, elem_bytes, d_workspace, ws_bytes, stream);
+}
+
+ipt_status ipt_0010(void *d_ptr, int64_t d0, int64_t d1, int64_t d2, int64_t d3, int elem_bytes,
+                    void *d_workspace, size_t ws_bytes, void *stream) {
+    int64_t b = 0;
+    if (d0 < 0 || d1 < 0 || !mul_ok(d0, d1, &b)) return IPT_ERR_INVALID_ARG;
+    return ipt_010(d_ptr, b, d2, d3, elem_bytes, d_workspace, ws_bytes, stream);
+}
+
+ipt_status ipt_0100(void *d_ptr, int64_t d0, int64_t d1, int64_t d2, int64_t d3, int elem_bytes,
+                    void *d_workspace, size_t ws_bytes, void *stream) {
+    return ipt_100(d_ptr, d0, d1, d2, d3, elem_bytes, d_workspace, ws_bytes, stream);
+}
+
+ipt_status ipt_1000(void *d_ptr, int64_t d0, int64_t d1, int64_t d2, int64_t d3, int elem_bytes,
+                    void *d_workspace, size_t ws_bytes, void *stream) {
+    int64_t s = 0;
+    if (d2 < 1 || d3 < 1 || !mul_ok(d2, d3, &s)) return IPT_ERR_INVALID_ARG;
+    return ipt_100(d_ptr, 1, d0, d1, s, elem_bytes, d_workspace, ws_bytes, stream);
+}
+
+// ------------------------------------------------- host-delegated transposition (Sec. 6)
+// the matrix is copied to the GPU (1), transposed in place there (2), and
+// copied back to the same host location (3).  Stage 1 (100!) spans the whole array and
+// cannot be split; stages 2 and 3 work on independent instances, so the
+// N' output panels are split into Q groups, each on its own stream: stage 2 + stage 3 +
+// device-to-host copy of the group overlap with the other groups' work (Fig. 5b).
+static ipt_status host_streams(int device, int q, cudaStream_t *out) {
+    static std::mutex mu;
+    static std::map<int, std::vector<cudaStream_t>> cache;
+    std::lock_guard<std::mutex> lk(mu);
+    auto &v = cache[device];
+    while ((int)v.size() < q) {
+        cudaStream_t s;
+        if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) {
+            cudaGetLastError();
+            return IPT_ERR_CUDA;
+        }
+        v.push_back(s);
+    }
+    for (int i = 0; i < q; ++i) out[i] = v[i];
+    return IPT_OK;
+}
+
+static size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+ipt_status ipt_transpose_host(void *h_ptr, int64_t M, int64_t N, int elem_bytes, int queues,
+                              void *d_buffer, size_t d_buffer_bytes, void *stream) {
+    int64_t bytes = 0;
+    ipt_status s = check_shape(M, N, elem_bytes, &bytes);
+    if (s) return s;
+    if ((s = check_ptr(h_ptr, elem_bytes))) return s;
+    if (queues < 1 || queues > 64) return IPT_ERR_INVALID_ARG;
+    if (M == 1 || N == 1) return IPT_OK;
+    const int device = current_device();
+    if (device < 0) return IPT_ERR_NO_DEVICE;
+    ipt_plan_t p;
+    if ((s = ipt_plan(M, N, elem_bytes, device, &p))) return s;
+    const int64_t Np = p.Np;
+    const int Q = (int)std::min<int64_t>(queues, Np);
+    StageDesc sd[3];
+    // workspace layout: [data | stage-1 flags | group 0 flags | group 1 flags | ...]
+    plan_stages(&p, nullptr, 1, bytes, sd);
+    size_t ws1 = p.variant[0] == IPT_VAR_CYCLE_GLOBAL ? cycle_ws_bytes(sd[0]) : 0;
+    std::vector<int64_t> g0(Q + 1);
+    for (int g = 0; g <= Q; ++g) g0[g] = Np * g / Q;
+    std::vector<size_t> wsg(Q, 0);
+    for (int g = 0; g < Q; ++g) {
+        StageDesc a = sd[1], b = sd[2];
+        a.inner = (g0[g + 1] - g0[g]) * p.Mp;
+        b.inner = g0[g + 1] - g0[g];
+        size_t w = 0;
+        if (p.variant[1] == IPT_VAR_CYCLE_GLOBAL) w = std::max(w, cycle_ws_bytes(a));
+        if (p.variant[2] == IPT_VAR_CYCLE_GLOBAL) w = std::max(w, cycle_ws_bytes(b));
+        wsg[g] = align256(w);
+    }
+    size_t need = align256((size_t)bytes) + align256(ws1);
+    for (size_t w : wsg) need += w;
+    char *dbuf = (char *)d_buffer;
+    cudaStream_t st = (cudaStream_t)stream;
+    if (!dbuf) {
+        void *w = nullptr;
+        if ((s = get_ws(device, (void *)((uintptr_t)stream ^ 0x1), need, &w))) return s;
+        dbuf = (char *)w;
+    } else if (d_buffer_bytes < need) {
+        return IPT_ERR_NO_MEMORY;
+    }
+    char *dws1 = dbuf + align256((size_t)bytes);
+    std::vector<char *> dwsg(Q);
+    char *cur = dws1 + align256(ws1);
+    for (int g = 0; g < Q; ++g) { dwsg[g] = cur; cur += wsg[g]; }
+    std::vector<cudaStream_t> qs(Q);
+    if ((s = host_streams(device, Q, qs.data()))) return s;
+
+    cudaError_t e = cudaMemcpyAsync(dbuf, h_ptr, (size_t)bytes, cudaMemcpyHostToDevice, st);
+    if (e != cudaSuccess) return cuda_status(e);
+    plan_stages(&p, dbuf, 1, bytes, sd);
+    if (p.variant[0] == IPT_VAR_CYCLE_GLOBAL) {
+        if ((e = launch_cycle_global(sd[0], dws1, st, device)) != cudaSuccess) return cuda_status(e);
+    }
+    cudaEvent_t ev1;
+    if ((e = cudaEventCreateWithFlags(&ev1, cudaEventDisableTiming)) != cudaSuccess) return cuda_status(e);
+    cudaEventRecord(ev1, st);
+    // panel q of the result (rows q*n .. q*n+n-1 of A^T) is the contiguous range
+    // [q*M*n, (q+1)*M*n) elements, both after stage 1 (N' x M x n) and after stage 3.
+    const int64_t panel = M * p.n * elem_bytes;
+    std::vector<cudaEvent_t> done(Q);
+    for (int g = 0; g < Q; ++g) {
+        cudaStream_t qs_g = qs[g];
+        cudaStreamWaitEvent(qs_g, ev1, 0);
+        char *gb = dbuf + g0[g] * panel;
+        const int64_t np_g = g0[g + 1] - g0[g];
+        StageDesc a = sd[1], b = sd[2];
+        a.base = gb; a.inner = np_g * p.Mp;
+        b.base = gb; b.inner = np_g;
+        if (p.variant[1] == IPT_VAR_TILE_ONCHIP) e = launch_tile_onchip(a, qs_g, device);
+        else if (p.variant[1] == IPT_VAR_CYCLE_GLOBAL) e = launch_cycle_global(a, dwsg[g], qs_g, device);
+        if (e != cudaSuccess) return cuda_status(e);
+        if (p.variant[2] == IPT_VAR_CYCLE_GLOBAL) e = launch_cycle_global(b, dwsg[g], qs_g, device);
+        if (e != cudaSuccess) return cuda_status(e);
+        e = cudaMemcpyAsync((char *)h_ptr + g0[g] * panel, gb, (size_t)(np_g * panel),
+                            cudaMemcpyDeviceToHost, qs_g);
+        if (e != cudaSuccess) return cuda_status(e);
+        cudaEventCreateWithFlags(&done[g], cudaEventDisableTiming);
+        cudaEventRecord(done[g], qs_g);
+        cudaStreamWaitEvent(st, done[g], 0);
+    }
+    e = cudaStreamSynchronize(st);
+    cudaEventDestroy(ev1);
+    for (auto d : done) cudaEventDestroy(d);
+    return cuda_status(e);
+}
+
+// -------------------------------------------------------------------- diagnostics
+const char *ipt_status_string(ipt_status s) {
+    switch (s) {
+        case IPT_OK: return "IPT_OK";
+        case IPT_ERR_INVALID_ARG: return "IPT_ERR_INVALID_ARG";
+        case IPT_ERR_UNSUPPORTED_ELEM: return "IPT_ERR_UNSUPPORTED_ELEM";
+        case IPT_ERR_MISALIGNED: return "IPT_ERR_MISALIGNED";
+        case IPT_ERR_NO_MEMORY: return "IPT_ERR_NO_MEMORY";
+        case IPT_ERR_CUDA: return "IPT_ERR_CUDA";
+        case IPT_ERR_NO_DEVICE: return "IPT_ERR_NO_DEVICE";
+    }
+    return "IPT_ERR_UNKNOWN";
+}
+
+uint64_t ipt_kernel_launch_count(void) { return g_launches.load(); }
+
+const char *ipt_version(void) { return "libipt 0.1 (sm_100a)"; }
+
+// Internal self-test hook (not in the ABI): the multiply-high division used by every
+// kernel's index map, evaluated on the host.
+uint64_t ipt__fastdiv(uint64_t n, uint64_t d) { return fdiv(n, make_fastdiv(d)); }
+
+}  // extern "C"

@@ -1,0 +1,92 @@
+// ipt_internal.h -- internal declarations shared by the libipt translation units.
+// Not part of the ABI (include/ipt.h is).  No oracle code is included or reachable.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stddef.h>
+
+#include "../../include/ipt.h"
+
+namespace ipt {
+
+// -------------------------------------------------------------- fast 64-bit division
+// Division by a run-time invariant divisor d via a multiply-high (Granlund & Montgomery,
+// "Division by invariant integers using multiplication", Fig. 4.1, N = 64):
+//   l = ceil(log2 d),  m = floor(2^64 (2^l - d) / d) + 1,
+//   t = mulhi(m, n),   q = (t + ((n - t) >> s1)) >> s2,  s1 = min(l, 1), s2 = max(l - 1, 0).
+// Exact for every 64-bit n.  Used for the index maps of every kernel so that no 64-bit
+// '%' or '/' appears in an inner loop (SURVEY.md Sec. 7 "64-bit index space").
+struct FastDiv {
+    uint64_t d;
+    uint64_t m;
+    uint32_t s1, s2;
+};
+
+FastDiv make_fastdiv(uint64_t d);  // host
+
+__host__ __device__ __forceinline__ uint64_t mulhi64(uint64_t a, uint64_t b) {
+#if defined(__CUDA_ARCH__)
+    return __umul64hi(a, b);
+#else
+    return (uint64_t)(((unsigned __int128)a * b) >> 64);
+#endif
+}
+
+__host__ __device__ __forceinline__ uint64_t fdiv(uint64_t n, const FastDiv &f) {
+    uint64_t t = mulhi64(n, f.m);
+    return (t + ((n - t) >> f.s1)) >> f.s2;
+}
+
+__host__ __device__ __forceinline__ void fdivmod(uint64_t n, const FastDiv &f, uint64_t &q,
+                                                 uint64_t &r) {
+    q = fdiv(n, f);
+    r = n - q * f.d;
+}
+
+// ------------------------------------------------------------------ stage descriptor
+// One elementary transposition P(batch, A, B, s): batch x [A x B x s] -> batch x [B x A x s]
+// (SURVEY.md R5).  The batch index T is split as T = to * inner + ti: item T starts at
+// base + to * ostride + ti * (A*B*s*eb) bytes, so that batched calls with an arbitrary
+// matrix stride fold into one launch.
+struct StageDesc {
+    char *base;
+    int64_t outer, inner;   // batch = outer * inner
+    int64_t ostride;        // bytes between outer items (>= inner * A*B*s*eb)
+    int64_t A, B, s;
+    int eb;                 // element bytes
+};
+
+// ---------------------------------------------------------------- kernel launchers
+// All launchers return cudaSuccess or the launch error; they only enqueue work.
+
+// Cycle following over super-elements with a global flag bitmap (PTTWAC over
+// super-elements, P:200-224 / SURVEY K5+K6).  `ws` must hold cycle_ws_bytes(desc).
+size_t cycle_ws_bytes(const StageDesc &d);
+cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, int device);
+
+// Whole-tile on-chip transposition (BS kernel, Fig. 1): s must be 1
+// and an A x B tile must fit in shared memory (tile_onchip_fits()).
+bool tile_onchip_fits(int64_t A, int64_t B, int eb, int device);
+// 0: does not fit, 1: generic element path, 2: 16-byte vector TMA path
+int tile_onchip_path(int64_t A, int64_t B, int eb, int device);
+cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device);
+
+// Device properties used by planner and launchers (cached).
+struct DevProps {
+    int sms;
+    int smem_optin;     // max dynamic shared memory per block (bytes)
+    int smem_per_sm;
+    int max_threads_sm;
+    int l2_bytes;
+    bool valid;
+};
+DevProps dev_props(int device);   // device < 0 -> nominal B200 values
+
+// Launch accounting (ipt_kernel_launch_count).
+void note_launch();
+
+// Environment-variable integer override (tuning knobs for tests / sweeps).
+long env_int(const char *name, long dflt);
+
+}  // namespace ipt

@@ -1,0 +1,146 @@
+"""CPU-only tests of the C ABI library (no GPU needed): it loads, exports every symbol
+include/ipt.h declares, validates arguments before touching a device, and the planner
+(Sec. 7.4) produces valid plans whose stage sequence (simulated with numpy) is the
+transpose.  No compute call is made here."""
+import ctypes
+import math
+import os
+import random
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_ppopp_sunggggh14_b200 as ipt
+from paper_conf_ppopp_sunggggh14_b200 import build as ipt_build
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _built():
+    ipt_build.build()
+
+
+def header_symbols():
+    txt = open(os.path.join(ROOT, "include", "ipt.h")).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(ipt_[a-z0-9_]+)\s*\(", txt)))
+
+
+def test_exports_every_header_symbol():
+    syms = header_symbols()
+    assert len(syms) >= 17
+    L = ctypes.CDLL(ipt.LIB_PATH)
+    for s in syms:
+        assert hasattr(L, s), s
+    # and the Python binding types every one of them
+    assert sorted(n for n, _, _ in ipt.ABI) == syms
+
+
+def test_library_is_sm100a():
+    out = os.popen(f"/usr/local/cuda/bin/cuobjdump --list-elf {ipt.LIB_PATH} 2>&1").read()
+    assert "sm_100a" in out, out
+
+
+def test_status_strings_and_version():
+    L = ipt.lib()
+    for code in range(7):
+        assert L.ipt_status_string(code).decode().startswith("IPT_")
+    assert "sm_100a" in ipt.version()
+
+
+def test_validation_before_device():
+    """Errors are returned before any launch (and without a GPU)."""
+    L = ipt.lib()
+    null = ctypes.c_void_p(0)
+    assert L.ipt_transpose(null, 4, 4, 4, null) == 1                       # NULL data
+    assert L.ipt_transpose(ctypes.c_void_p(256), 4, 4, 3, null) == 2        # elem 3
+    assert L.ipt_transpose(ctypes.c_void_p(258), 4, 4, 4, null) == 3        # misaligned
+    assert L.ipt_transpose(ctypes.c_void_p(256), 0, 4, 4, null) == 1        # M < 1
+    assert L.ipt_transpose(ctypes.c_void_p(256), 2**40, 2**40, 4, null) == 1  # overflow
+    assert L.ipt_transpose(ctypes.c_void_p(256), 1, 77, 4, null) == 0       # 1 x N: no-op
+    assert L.ipt_transpose(ctypes.c_void_p(256), 77, 1, 8, null) == 0       # M x 1: no-op
+    assert L.ipt_100(ctypes.c_void_p(256), 1, 0, 3, 1, 4, null, 0, null) == 1
+    assert L.ipt_100(ctypes.c_void_p(256), 0, 3, 3, 1, 4, null, 0, null) == 0  # empty batch
+    assert L.ipt_transpose_batched(ctypes.c_void_p(256), 2, 4, 4, 4, 4, null) == 1  # stride too small
+    p = ipt.Plan()
+    assert L.ipt_plan_with_tiles(12, 10, 5, 5, 4, -1, ctypes.byref(p)) == 1   # 5 does not divide 12
+
+
+def test_fastdiv_exact():
+    """The multiply-high division used by every kernel's index map (host evaluation)."""
+    L = ipt.lib()
+    rnd = random.Random(3)
+    ds = [1, 2, 3, 7, 25, 127, 128, 129, 1800, 7200, 12345678, 2**31 - 1, 2**32 + 15,
+          2**63 - 25, 2**63, 2**64 - 1]
+    ns = [0, 1, 2, 3, 2**32 - 1, 2**32, 2**63 - 1, 2**63, 2**64 - 1, 2**64 - 2]
+    for d in ds:
+        for n in ns + [rnd.randrange(2**64) for _ in range(200)] + [rnd.randrange(10**7) for _ in range(50)]:
+            assert L.ipt__fastdiv(n, d) == n // d, (n, d)
+
+
+# ----------------------------------------------------------------------------- planner
+def _np_stages(a, M, N, m, n):
+    Mp, Np = M // m, N // n
+    a = a.reshape(M, Np, n).transpose(1, 0, 2).reshape(-1)            # 100!
+    a = a.reshape(Np, Mp, m, n).transpose(0, 1, 3, 2).reshape(-1)     # 0010!
+    a = a.reshape(Np, Mp, n, m).transpose(0, 2, 1, 3).reshape(-1)     # 0100!
+    return a
+
+
+SWEEP = [(1800, 7200), (7200, 1800), (5100, 2500), (4000, 3200), (3300, 3900), (2500, 5100),
+         (1024, 16384), (4096, 4096), (8192, 2048), (9998, 4096), (9797, 13081), (14803, 1024),
+         (19997, 1024), (1021, 4093), (1009, 7001), (10007, 19997), (1_000_000, 256),
+         (20000, 30000), (4096, 3000), (5, 3), (64, 64), (2, 2)]
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+def test_plan_valid(eb):
+    for (M, N) in SWEEP:
+        p = ipt.plan(M, N, eb)
+        assert p.M == M and p.N == N and M % p.m == 0 and N % p.n == 0
+        assert p.Mp * p.m == M and p.Np * p.n == N
+        v = [ipt.VARIANTS[x] for x in p.variant]
+        # identity stages exactly when a swapped dimension is 1
+        assert (v[0] == "identity") == (p.Np == 1)
+        assert (v[1] == "identity") == (p.m == 1 or p.n == 1)
+        assert (v[2] == "identity") == (p.Mp == 1 or p.n == 1)
+        assert p.n_stages == sum(x != "identity" for x in v)
+        # deterministic
+        q = ipt.plan(M, N, eb)
+        assert (q.m, q.n, list(q.variant)) == (p.m, p.n, list(p.variant))
+
+
+def test_plan_stage_simulation_is_transpose():
+    rnd = random.Random(5)
+    shapes = [(rnd.randint(1, 90), rnd.randint(1, 90)) for _ in range(40)] + [(5, 3), (97, 89)]
+    for (M, N) in shapes:
+        p = ipt.plan(M, N, 4)
+        a = np.arange(M * N, dtype=np.uint32)
+        assert np.array_equal(_np_stages(a, M, N, p.m, p.n), a.reshape(M, N).T.reshape(-1))
+
+
+def test_plan_overhead_below_paper_bound():
+    """flag bits ~ one per super-element; < 0.1% with m, n in [50, 100]."""
+    for (M, N) in [(7200, 1800), (1800, 7200), (4000, 3200), (20000, 20000)]:
+        p = ipt.plan(M, N, 4, m=None, n=None)
+        data = M * N * 4
+        assert p.workspace_bytes < 0.001 * data, (M, N, p.workspace_bytes)
+    p = ipt.plan(7200, 1800, 4, m=60, n=60)
+    assert p.workspace_bytes < 0.001 * 7200 * 1800 * 4
+
+
+def test_plan_prefers_vector_tiles_on_large_f32():
+    """Sec. 7.4 pruning: big super-elements for stages 1/3, tile on chip for stage 2."""
+    for (M, N) in [(7200, 1800), (16384, 16384), (20000, 20000)]:
+        p = ipt.plan(M, N, 4)
+        assert p.n * 4 >= 256 and p.m * 4 >= 256
+        assert ipt.VARIANTS[p.variant[1]] == "tile_onchip"
+        assert p.n_stages == 3
+
+
+def test_workspace_batch_scales():
+    p = ipt.plan(4096, 3000, 4)
+    w1, w8 = ipt.workspace_bytes(p, 1), ipt.workspace_bytes(p, 8)
+    assert w8 > w1 and w8 <= 8 * w1 + 256

@@ -1,0 +1,366 @@
+"""GPU parity: libipt's CUDA kernels (through the C ABI) vs the CPU oracle, bit-exact.
+
+Small/medium sizes span many tiles, chains and ragged tails and are compared element by
+element with the oracle's output on the same seeded input.  Full BASELINE sizes are run
+in the bench's launch configuration and checked (a) on sampled outputs computed one by
+one by the oracle's Eq. (1) and the generator, and (b) on every element through the
+transposition's definition A^T(j, i) = A(i, j) evaluated with torch index arithmetic.
+"""
+import os
+import random
+
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+import paper_conf_ppopp_sunggggh14_b200 as ipt  # noqa: E402
+from inputs import seeded  # noqa: E402
+from oracle import oracle  # noqa: E402
+
+_TDT = {1: torch.uint8, 2: torch.int16, 4: torch.int32, 8: torch.int64}
+_NDT = {1: np.uint8, 2: np.int16, 4: np.int32, 8: np.int64}
+
+
+def to_dev(a: np.ndarray, eb: int):
+    if eb == 16:
+        return torch.from_numpy(a.view(np.int64).copy()).cuda()
+    return torch.from_numpy(a.view(_NDT[eb]).copy()).cuda()
+
+
+def to_np(t, eb: int):
+    a = t.cpu().numpy()
+    if eb == 16:
+        return a.view(np.uint64)
+    return a.view(oracle.dtype_for(eb))
+
+
+def gen(n_elems: int, eb: int, seed=seeded.SEED):
+    if eb == 16:
+        return seeded.values_np(np.arange(2 * n_elems), 8, seed)
+    return seeded.values_np(np.arange(n_elems), eb, seed)
+
+
+def oracle_P(a, batch, A, B, s, eb):
+    if eb == 16:  # 16-byte elements = super-elements of two 8-byte words
+        return oracle.permute_inplace(a, batch, A, B, 2 * s)
+    return oracle.permute_inplace(a, batch, A, B, s)
+
+
+@pytest.fixture(autouse=True)
+def _env_clean(monkeypatch):
+    for k in list(os.environ):
+        if k.startswith("IPT_"):
+            monkeypatch.delenv(k, raising=False)
+    yield
+
+
+# -------------------------------------------------------------- elementary: 100! / 0100!
+@pytest.mark.parametrize("eb", [4, 8])
+def test_ipt_100_random_shapes(eb):
+    rnd = random.Random(100 + eb)
+    for _ in range(60):
+        batch = rnd.choice([1, 1, 2, 3, 5])
+        A, B = rnd.randint(1, 70), rnd.randint(1, 70)
+        s = rnd.choice([1, 2, 3, 4, 7, 8, 16, 25, 32, 50, 64, 100, 129, 200, 333])
+        a = gen(batch * A * B * s, eb)
+        t = to_dev(a, eb)
+        ipt.ipt_100_(t, batch, A, B, s)
+        ref = oracle_P(a.copy(), batch, A, B, s, eb)
+        assert np.array_equal(to_np(t, eb), ref), (batch, A, B, s, eb)
+
+
+@pytest.mark.parametrize("eb", [1, 2, 16])
+def test_ipt_100_other_elem_sizes(eb):
+    rnd = random.Random(7 + eb)
+    for _ in range(25):
+        batch, A, B, s = rnd.randint(1, 3), rnd.randint(1, 40), rnd.randint(1, 40), rnd.choice([1, 3, 5, 16, 33])
+        a = gen(batch * A * B * s, eb)
+        t = to_dev(a, eb)
+        ipt.ipt_100_(t, batch, A, B, s, elem_bytes=eb)
+        ref = oracle_P(a.copy(), batch, A, B, s, eb)
+        assert np.array_equal(to_np(t, eb), ref), (batch, A, B, s, eb)
+
+
+def test_ipt_0100_and_1000_definitions():
+    d0, d1, d2, d3 = 3, 7, 5, 24
+    a = gen(d0 * d1 * d2 * d3, 4)
+    t = to_dev(a, 4)
+    ipt.ipt_0100_(t, d0, d1, d2, d3)
+    ref = oracle.permute_inplace(a.copy(), d0, d1, d2, d3)
+    assert np.array_equal(to_np(t, 4), ref)
+    t = to_dev(a, 4)
+    ipt.ipt_1000_(t, d0, d1, d2, d3)
+    ref = oracle.permute_inplace(a.copy(), 1, d0, d1, d2 * d3)
+    assert np.array_equal(to_np(t, 4), ref)
+
+
+@pytest.mark.parametrize("G,R,maxvec", [(32, 1, 128), (16, 2, 128), (8, 4, 128), (4, 4, 128),
+                                        (32, 4, 128), (32, 2, 7), (32, 1, 3)])
+def test_ipt_100_forced_walker_shapes(monkeypatch, G, R, maxvec):
+    """Every walker shape (lanes per walker G, vectors per lane R) and super-element
+    chunking gives identical bytes."""
+    monkeypatch.setenv("IPT_CYC_G", str(G))
+    monkeypatch.setenv("IPT_CYC_R", str(R))
+    monkeypatch.setenv("IPT_CYC_MAXVEC", str(maxvec))
+    for (batch, A, B, s) in [(1, 61, 47, 8), (2, 33, 20, 12), (1, 128, 96, 4), (3, 17, 19, 2)]:
+        a = gen(batch * A * B * s, 4)
+        t = to_dev(a, 4)
+        ipt.ipt_100_(t, batch, A, B, s)
+        assert np.array_equal(to_np(t, 4), oracle.permute_inplace(a.copy(), batch, A, B, s)), (G, R, batch, A, B, s)
+
+
+# -------------------------------------------------------------- elementary: 010! / 0010!
+@pytest.mark.parametrize("eb", [4, 8, 16])
+def test_ipt_010_tile_fast_path(eb):
+    V = 16 // eb
+    rnd = random.Random(eb)
+    for _ in range(30):
+        batch = rnd.randint(1, 400)
+        A, B = V * rnd.randint(1, 40), V * rnd.randint(1, 40)
+        a = gen(batch * A * B, eb)
+        t = to_dev(a, eb)
+        ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+        ref = oracle_P(a.copy(), batch, A, B, 1, eb)
+        assert np.array_equal(to_np(t, eb), ref), (batch, A, B, eb)
+
+
+@pytest.mark.parametrize("eb", [1, 2, 4, 8, 16])
+def test_ipt_010_tile_generic_path(eb):
+    rnd = random.Random(50 + eb)
+    for _ in range(20):
+        batch, A, B = rnd.randint(1, 200), rnd.randint(1, 61), rnd.randint(1, 61)
+        a = gen(batch * A * B, eb)
+        t = to_dev(a, eb)
+        ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+        ref = oracle_P(a.copy(), batch, A, B, 1, eb)
+        assert np.array_equal(to_np(t, eb), ref), (batch, A, B, eb)
+
+
+def test_ipt_010_large_tile_falls_back_to_cycles():
+    """A tile larger than shared memory uses cycle following (s = 1)."""
+    batch, A, B = 3, 301, 257        # 309 KB f32 tiles
+    a = gen(batch * A * B, 4)
+    t = to_dev(a, 4)
+    ipt.ipt_0010_(t, 1, batch, A, B)
+    assert np.array_equal(to_np(t, 4), oracle.permute_inplace(a.copy(), batch, A, B, 1))
+
+
+def test_ipt_010_forced_generic(monkeypatch):
+    monkeypatch.setenv("IPT_TILE_GENERIC", "1")
+    batch, A, B = 37, 64, 48
+    a = gen(batch * A * B, 4)
+    t = to_dev(a, 4)
+    ipt.ipt_010_(t, batch, A, B)
+    assert np.array_equal(to_np(t, 4), oracle.permute_inplace(a.copy(), batch, A, B, 1))
+
+
+# ------------------------------------------------------------------- full transposition
+SMALL_SHAPES = [(5, 3), (3, 5), (2, 2), (64, 64), (100, 36), (36, 100), (97, 89), (89, 97),
+                (1021, 13), (13, 1021), (256, 1000), (480, 360), (720, 180), (1, 1000),
+                (1000, 1), (331, 337), (128, 1024), (600, 999), (2 * 499, 1024)]
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+def test_transpose_small_shapes(eb):
+    for (M, N) in SMALL_SHAPES:
+        a = seeded.matrix_np(M, N, eb)
+        t = to_dev(a, eb)
+        out = ipt.transpose_(t, M, N)
+        assert tuple(out.shape) == (N, M)
+        ref = oracle.transpose_inplace(a.copy(), M, N)
+        assert np.array_equal(to_np(t, eb), ref), (M, N, eb)
+
+
+@pytest.mark.parametrize("eb", [1, 2, 16])
+def test_transpose_other_elem_sizes(eb):
+    for (M, N) in [(5, 3), (64, 48), (97, 89), (300, 120)]:
+        a = gen(M * N, eb)
+        t = to_dev(a, eb)
+        ipt.transpose_(t, M, N, elem_bytes=eb)
+        ref = oracle_P(a.copy(), 1, M, N, 1, eb)
+        assert np.array_equal(to_np(t, eb), ref), (M, N, eb)
+
+
+def test_plan_independence_all_tilings():
+    """Every valid (m, n) gives identical bytes."""
+    M, N = 120, 72
+    a = seeded.matrix_np(M, N, 4)
+    ref = oracle.transpose_inplace(a.copy(), M, N)
+    divs = lambda x: [d for d in range(1, x + 1) if x % d == 0]
+    for m in divs(M):
+        for n in divs(N):
+            p = ipt.plan(M, N, 4, m=m, n=n)
+            t = to_dev(a, 4)
+            ipt.transpose_(t, M, N, plan_=p)
+            assert np.array_equal(to_np(t, 4), ref), (m, n)
+
+
+def test_random_bits_and_double_transpose():
+    for eb in (4, 8):
+        M, N = 777, 360
+        a = seeded.random_bits_np(M * N, eb, seed=9)
+        t = to_dev(a, eb)
+        ipt.transpose_(t, M, N)
+        assert np.array_equal(to_np(t, eb), a.reshape(M, N).T.reshape(-1))
+        ipt.transpose_(t, N, M)
+        assert np.array_equal(to_np(t, eb), a)
+
+
+def test_user_workspace_and_events():
+    M, N = 1800, 720
+    p = ipt.plan(M, N, 4, device=0)
+    ws = torch.empty(ipt.workspace_bytes(p, 1), dtype=torch.uint8, device="cuda")
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+    for e in evs:
+        e.record()
+    a = seeded.matrix_np(M, N, 4)
+    t = to_dev(a, 4)
+    ipt.transpose_(t, M, N, plan_=p, workspace=ws, events=evs)
+    torch.cuda.synchronize()
+    assert np.array_equal(to_np(t, 4), oracle.transpose_inplace(a.copy(), M, N))
+    assert all(evs[i].elapsed_time(evs[i + 1]) >= 0 for i in range(3))
+
+
+def test_workspace_too_small_rejected():
+    p = ipt.plan(1800, 720, 4, device=0)
+    ws = torch.empty(16, dtype=torch.uint8, device="cuda")
+    t = torch.zeros(1800 * 720, dtype=torch.int32, device="cuda")
+    with pytest.raises(ipt.IptError, match="NO_MEMORY"):
+        ipt.transpose_(t, 1800, 720, plan_=p, workspace=ws)
+
+
+def test_cpu_tensor_refused():
+    with pytest.raises(ipt.IptError):
+        ipt.transpose_(torch.zeros(12, dtype=torch.int32), 3, 4)
+
+
+def test_native_kernels_launched():
+    before = ipt.kernel_launch_count()
+    t = to_dev(seeded.matrix_np(720, 1800, 4), 4)
+    ipt.transpose_(t, 720, 1800)
+    torch.cuda.synchronize()
+    assert ipt.kernel_launch_count() - before == ipt.plan(720, 1800, 4, device=0).n_stages
+
+
+# -------------------------------------------------------------------------------- batch
+def test_batched_with_stride():
+    count, M, N = 7, 360, 96
+    stride = M * N + 40
+    a = seeded.values_np(np.arange(count * stride), 4)
+    t = to_dev(a, 4)
+    ipt.transpose_batched_(t, count, M, N, stride_elems=stride)
+    ref = a.copy()
+    for i in range(count):
+        seg = ref[i * stride: i * stride + M * N]
+        oracle.transpose_inplace(seg, M, N)
+    assert np.array_equal(to_np(t, 4), ref)
+
+
+# ------------------------------------------------------------------ race stress (T6)
+def test_stress_varied_occupancy(monkeypatch):
+    """Repeat with different persistent-grid sizes and walker shapes so chains
+    interleave differently; every run must be bit-exact."""
+    M, N = 1200, 1800
+    a = seeded.matrix_np(M, N, 4)
+    ref = oracle.transpose_inplace(a.copy(), M, N)
+    rnd = random.Random(1)
+    for it in range(40):
+        monkeypatch.setenv("IPT_CYC_BLOCKS_PER_SM", str(rnd.choice([1, 2, 3, 8])))
+        monkeypatch.setenv("IPT_CYC_REFRESH", str(rnd.choice([0, 1])))
+        m, n = rnd.choice([(120, 120), (60, 90), (40, 200), (300, 24), (8, 1800)])
+        t = to_dev(a, 4)
+        ipt.transpose_(t, M, N, plan_=ipt.plan(M, N, 4, m=m, n=n))
+        assert np.array_equal(to_np(t, 4), ref), (it, m, n)
+
+
+# ------------------------------------------------------- full BASELINE sizes (sampled)
+def _check_full(t, M, N, eb, t_idx=0, nsamp=20000, seed=0):
+    """(a) sampled outputs via the oracle's Eq. (1), one by one; (b) every element via the
+    definition with torch index arithmetic (on the device)."""
+    rnd = random.Random(seed)
+    n = M * N
+    ks = [rnd.randrange(n) for _ in range(nsamp)] + [0, 1, n - 2, n - 1]
+    dst = torch.tensor([oracle.eq1_dest(k, M, N) for k in ks], device=t.device)
+    exp = seeded.values_torch_sample(torch.tensor(ks, device=t.device) + t_idx * n, eb)
+    got = t.view(-1)[:n][dst]
+    assert torch.equal(got, exp.to(t.dtype))
+    # whole array, in chunks: position p = j*M + i holds v(i*N + j)
+    CH = 1 << 27
+    for p0 in range(0, n, CH):
+        p = torch.arange(p0, min(n, p0 + CH), device=t.device, dtype=torch.int64)
+        j, i = p // M, p % M
+        exp = seeded.values_torch_sample(i * N + j + t_idx * n, eb)
+        assert torch.equal(t.view(-1)[p0:p0 + p.numel()], exp.to(t.dtype)), p0
+
+
+@pytest.mark.parametrize("M,N,eb", [(1800, 7200, 4), (7200, 1800, 4)])
+def test_full_config_C1_vs_oracle(M, N, eb):
+    a = seeded.matrix_np(M, N, eb)
+    t = to_dev(a, eb)
+    ipt.transpose_(t, M, N)
+    assert np.array_equal(to_np(t, eb), oracle.transpose_inplace(a.copy(), M, N))
+
+
+SWEEP_FULL = [(7200, 18000), (18000, 7200), (16384, 16384), (12800, 15000), (19200, 10000),
+              (9998, 12288), (14803, 8192), (20000, 20000), (5100, 2500), (4000, 3200),
+              (3300, 3900), (2500, 5100), (1021, 4093), (19997, 1024)]
+
+
+@pytest.mark.parametrize("M,N", SWEEP_FULL)
+def test_full_config_sweep_f32(M, N):
+    t = torch.empty(M * N, dtype=torch.int32, device="cuda")
+    seeded.fill_device_(t, M, N, 4)
+    ipt.transpose_(t, M, N)
+    _check_full(t, M, N, 4)
+
+
+def test_full_config_C3_skinny():
+    M, N = 1_000_000, 256
+    t = torch.empty(M * N, dtype=torch.int32, device="cuda")
+    seeded.fill_device_(t, M, N, 4)
+    ipt.transpose_(t, M, N)
+    _check_full(t, M, N, 4)
+
+
+def test_full_config_C4_large_f64():
+    M, N = 20000, 30000
+    t = torch.empty(M * N, dtype=torch.int64, device="cuda")
+    seeded.fill_device_(t, M, N, 8)
+    ipt.transpose_(t, M, N)
+    _check_full(t, M, N, 8)
+    del t
+    torch.cuda.empty_cache()
+
+
+def test_full_config_C5_batch_sampled():
+    count, M, N = 64, 4096, 3000      # one GPU's shard at G = 8
+    t = torch.empty(count * M * N, dtype=torch.int32, device="cuda")
+    seeded.fill_device_(t, M, N, 4, count=count)
+    ipt.transpose_batched_(t, count, M, N)
+    for ti in (0, 1, count // 2, count - 1):
+        _check_full(t[ti * M * N:(ti + 1) * M * N], M, N, 4, t_idx=ti, nsamp=2000, seed=ti)
+    del t
+    torch.cuda.empty_cache()
+
+
+def test_prime_both_scalar_fallback():
+    M, N = 10007, 19997
+    t = torch.empty(M * N, dtype=torch.int32, device="cuda")
+    seeded.fill_device_(t, M, N, 4)
+    ipt.transpose_(t, M, N)
+    _check_full(t, M, N, 4, nsamp=5000)
+
+
+# ------------------------------------------------------ host-delegated scheme (Sec. 6)
+@pytest.mark.parametrize("queues", [1, 3, 8])
+def test_transpose_host_queues(queues):
+    for (M, N) in [(1800, 7200), (360, 1000), (97, 89)]:
+        a = seeded.matrix_np(M, N, 4)
+        h = torch.from_numpy(a.view(np.int32).copy()).pin_memory()
+        out = ipt.transpose_host_(h, M, N, queues=queues)
+        assert tuple(out.shape) == (N, M)
+        ref = oracle.transpose_inplace(a.copy(), M, N)
+        assert np.array_equal(h.numpy().view(np.uint32), ref), (M, N, queues)

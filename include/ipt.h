@@ -174,6 +174,9 @@ const char *ipt_status_string(ipt_status s);
 /* Number of libipt kernels launched by this process so far (all devices). */
 uint64_t ipt_kernel_launch_count(void);
 
+/* Description of the CUDA error behind the calling thread's last IPT_ERR_CUDA. */
+const char *ipt_last_cuda_error(void);
+
 /* Library version string. */
 const char *ipt_version(void);
 

@@ -76,6 +76,7 @@ ABI = [
     ("ipt_1000", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
     ("ipt_status_string", ctypes.c_char_p, [_int]),
     ("ipt_kernel_launch_count", ctypes.c_uint64, []),
+    ("ipt_last_cuda_error", ctypes.c_char_p, []),
     ("ipt_version", ctypes.c_char_p, []),
 ]
 
@@ -101,7 +102,10 @@ def lib():
 
 def _check(rc: int, what: str):
     if rc != IPT_OK:
-        raise IptError(f"{what}: {lib().ipt_status_string(rc).decode()}")
+        msg = lib().ipt_status_string(rc).decode()
+        if msg == "IPT_ERR_CUDA":
+            msg += f" ({lib().ipt_last_cuda_error().decode()})"
+        raise IptError(f"{what}: {msg}")
 
 
 def _stream_ptr(stream):

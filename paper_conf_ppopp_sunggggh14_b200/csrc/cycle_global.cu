@@ -51,6 +51,8 @@ struct CycParams {
     uint32_t *flags;
     unsigned long long *counter;
     int refresh;        // re-read the flag word after a chain ends before the next start
+    uint32_t zero;      // always 0 at run time; opaque to the compiler (see dep_zero use)
+    int fence;          // 1: PTX-model fences on both sides of the claim protocol
 };
 
 enum : int { M_FETCH = 0, M_SCAN = 1, M_START = 2, M_CHAIN = 3, M_REFRESH = 4, M_DONE = 5 };
@@ -136,7 +138,10 @@ __global__ void __launch_bounds__(256) cycle_global_kernel(const CycParams p) {
             fdivmod(k, p.divB, q, r);
             tgt = r * p.A + q;                         // Eq. (1) on super-element offsets
         }
-        const bool back_home = (mode == M_CHAIN) && (tgt == k0);   // cycle closed at our start
+        // Cycle closed at our own start x: x must still be CLAIMED (another walker carrying
+        // A[prev(x)] -- the start walker of prev(x) -- may race for it), but its backup is
+        // the value this walker already delivered, so it is not re-read.
+        const bool back_home = (mode == M_CHAIN) && (tgt == k0);
         const uint64_t ut = ubase + tgt * p.nchunk;    // flag index of the target unit
         const uint32_t bit = 1u << (ut & 31);
         char *addr = item + tgt * p.S;
@@ -149,22 +154,26 @@ __global__ void __launch_bounds__(256) cycle_global_kernel(const CycParams p) {
             }
         }
         uint32_t old = 0;
-        if (mode == M_CHAIN && !back_home && gl == 0) old = atom_or_u32(p.flags + (ut >> 5), bit);
+        if (mode == M_CHAIN && gl == 0)
+            old = p.fence ? atom_or_acq_u32(p.flags + (ut >> 5), bit)
+                          : atom_or_u32(p.flags + (ut >> 5), bit);
         uint32_t fw = 0;
         if (mode == M_START) {
+            if (p.fence) fence_acq_rel_gpu();
             uint32_t acc = 0;
 #pragma unroll
             for (int r = 0; r < R; ++r) {
                 const int v = gl + r * G;
                 if (v < nv) acc |= fold(in[r]);
             }
-            fw = ld_relaxed_u32(p.flags + (ut >> 5) + dep_zero(acc));
+            fw = ld_relaxed_u32(p.flags + (ut >> 5) + (acc & p.zero));
         } else if (mode == M_REFRESH) {
             fw = ld_relaxed_u32(p.flags + word);
         }
 
         // ------------------------------------------------------------------- resolve
         old = __shfl_sync(FULL, old, g0);
+        __syncwarp();   // orders lane 0's (acquire) claim before the other lanes' stores
         const unsigned seen = __ballot_sync(FULL, mode == M_START && (fw & bit));
         const uint32_t fw0 = __shfl_sync(FULL, fw, g0);
         if (mode == M_START) {
@@ -177,7 +186,7 @@ __global__ void __launch_bounds__(256) cycle_global_kernel(const CycParams p) {
                 mode = M_CHAIN;
             }
         } else if (mode == M_CHAIN) {
-            if (back_home || !(old & bit)) {
+            if (!(old & bit)) {
 #pragma unroll
                 for (int r = 0; r < R; ++r) {
                     const int v = gl + r * G;
@@ -339,6 +348,8 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
     p.counter = (unsigned long long *)ws;
     p.flags = (uint32_t *)((char *)ws + 256);
     p.refresh = (int)env_int("IPT_CYC_REFRESH", 1);
+    p.zero = 0;
+    p.fence = (int)env_int("IPT_CYC_FENCE", 1);
     cudaError_t e = cudaMemsetAsync(ws, 0, 256 + p.nwords * 4, st);
     if (e != cudaSuccess) return e;
     return fn(p, st, device);

@@ -149,8 +149,11 @@ ipt_status get_ws(int device, void *stream, size_t need, void **out) {
     return IPT_OK;
 }
 
+thread_local cudaError_t g_last_cuda = cudaSuccess;
+
 ipt_status cuda_status(cudaError_t e) {
     if (e == cudaSuccess) return IPT_OK;
+    g_last_cuda = e;
     cudaGetLastError();
     return IPT_ERR_CUDA;
 }
@@ -524,6 +527,8 @@ const char *ipt_status_string(ipt_status s) {
 }
 
 uint64_t ipt_kernel_launch_count(void) { return g_launches.load(); }
+
+const char *ipt_last_cuda_error(void) { return cudaGetErrorString(g_last_cuda); }
 
 const char *ipt_version(void) { return "libipt 0.1 (sm_100a)"; }
 

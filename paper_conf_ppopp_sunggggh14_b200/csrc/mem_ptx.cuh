@@ -91,6 +91,17 @@ __device__ __forceinline__ uint32_t atom_or_u32(uint32_t *p, uint32_t bits) {
     return old;
 }
 
+__device__ __forceinline__ uint32_t atom_or_acq_u32(uint32_t *p, uint32_t bits) {
+    uint32_t old;
+    asm volatile("atom.acquire.gpu.global.or.b32 %0, [%1], %2;"
+                 : "=r"(old) : "l"(p), "r"(bits) : "memory");
+    return old;
+}
+
+__device__ __forceinline__ void fence_acq_rel_gpu() {
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+}
+
 // ------------------------------------------------------------ mbarrier / bulk copy
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return (uint32_t)__cvta_generic_to_shared(p);

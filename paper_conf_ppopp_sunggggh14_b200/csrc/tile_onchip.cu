@@ -221,7 +221,10 @@ int occupancy(K kern, size_t smem, int device) {
     auto it = cache.find(key);
     if (it != cache.end()) return it->second;
     int n = 0;
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    // one attribute value per kernel: the device maximum (a lower value set for one
+    // shape would make a later, larger launch fail)
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         dev_props(device).smem_optin);
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, 256, smem) != cudaSuccess) n = 1;
     if (n < 1) n = 1;
     cache[key] = n;

@@ -72,6 +72,28 @@ def test_ipt_100_random_shapes(eb):
         assert np.array_equal(to_np(t, eb), ref), (batch, A, B, s, eb)
 
 
+@pytest.mark.parametrize("batch,A,s", [(128, 128, 128), (16, 128, 128), (128, 64, 128),
+                                       (128, 128, 4), (128, 128, 1), (1, 1024, 4), (1, 2048, 1),
+                                       (64, 200, 32)])
+def test_ipt_100_square(batch, A, s):
+    """Square A x A super-element matrices: every cycle has length 2 and closes at its
+    start, the case that exposed the unclaimed cycle-close race (tools/protocol_sim.py)."""
+    n = batch * A * A * s
+    t = torch.empty(n, dtype=torch.int32, device="cuda")
+    seeded.fill_device_(t, n, 1, 4)
+    ref = t.clone()
+    for _ in range(2):
+        ipt.ipt_100_(t, batch, A, A, s)
+        ref = ref.view(batch, A, A, s).permute(0, 2, 1, 3).contiguous().view(-1)
+        assert torch.equal(t, ref)
+    # sampled against the oracle's own Eq. (1) as well
+    a = gen(min(n, 3 * A * A * s), 4)
+    tt = to_dev(a, 4)
+    b3 = len(a) // (A * A * s)
+    ipt.ipt_100_(tt, b3, A, A, s)
+    assert np.array_equal(to_np(tt, 4), oracle.permute_inplace(a.copy(), b3, A, A, s))
+
+
 @pytest.mark.parametrize("eb", [1, 2, 16])
 def test_ipt_100_other_elem_sizes(eb):
     rnd = random.Random(7 + eb)

@@ -53,6 +53,9 @@ struct CycParams {
     int refresh;        // re-read the flag word after a chain ends before the next start
     uint32_t zero;      // always 0 at run time; opaque to the compiler (see dep_zero use)
     int fence;          // 1: PTX-model fences on both sides of the claim protocol
+    int pf;             // chain look-ahead depth (L2 prefetch of the next targets)
+    uint64_t wstride;   // start-order scramble (coprime to nwords)
+    FastDiv divNwords;
 };
 
 enum : int { M_FETCH = 0, M_SCAN = 1, M_START = 2, M_CHAIN = 3, M_REFRESH = 4, M_DONE = 5 };
@@ -87,13 +90,24 @@ __global__ void __launch_bounds__(256) cycle_global_kernel(const CycParams p) {
                 unsigned long long wb = 0;
                 if (lane == leader) wb = atomicAdd(p.counter, (unsigned long long)__popc(need));
                 wb = __shfl_sync(FULL, wb, leader);
-                const uint64_t mine = wb + __popc(need & ((1u << g0) - 1u));
+                uint64_t mine = wb + __popc(need & ((1u << g0) - 1u));
+                const bool have = mine < p.nwords;
+                // Start order: fetch i scans flag word (i * wstride) mod nwords.  For a
+                // batch of small independent matrices wstride ~ words per matrix, so the
+                // start frontier advances through all matrices at once (like one big
+                // matrix) instead of bursting through one at a time, which keeps chains
+                // long and PTTWAC's redundant start reads low.
+                if (have && p.wstride != 1) {
+                    uint64_t q, r;
+                    fdivmod(mine * p.wstride, p.divNwords, q, r);
+                    mine = r;
+                }
                 uint32_t fw = 0;
-                if (mode == M_FETCH && mine < p.nwords) fw = ld_relaxed_u32(p.flags + mine);
+                if (mode == M_FETCH && have) fw = ld_relaxed_u32(p.flags + mine);
                 fw = __shfl_sync(FULL, fw, g0);
                 if (mode == M_FETCH) {
                     word = mine;
-                    if (word >= p.nwords) {
+                    if (!have) {
                         mode = M_DONE;
                     } else {
                         cw = fw;
@@ -151,6 +165,24 @@ __global__ void __launch_bounds__(256) cycle_global_kernel(const CycParams p) {
             for (int r = 0; r < R; ++r) {
                 const int v = gl + r * G;
                 if (v < nv) in[r] = ld_cg<W>(addr + (size_t)v * W);
+            }
+            // Look-ahead: the chain's next positions are known from Eq. (1) alone, so the
+            // lines of the next `pf` targets are prefetched into L2 now; their backup reads
+            // (issued in later rounds, only by whoever claims them) then hit L2 instead of
+            // paying a DRAM round trip per chain step.  No data is consumed early, so the
+            // claim protocol is unchanged; a prefetch is wasted only at a chain's true end
+            // (the winner of a lost claim walks the same targets).
+            uint64_t la = tgt;
+            for (int j = 0; j < p.pf; ++j) {
+                uint64_t q, r;
+                fdivmod(la, p.divB, q, r);
+                la = r * p.A + q;
+                if (la == k0) break;
+                const uintptr_t lo = (uintptr_t)(item + la * p.S);
+                const uintptr_t first = lo & ~(uintptr_t)127;
+                const uintptr_t last = (lo + (uintptr_t)nv * W - 1) & ~(uintptr_t)127;
+                for (uintptr_t line = first + (uintptr_t)gl * 128; line <= last; line += (uintptr_t)G * 128)
+                    prefetch_l2((const void *)line);
             }
         }
         uint32_t old = 0;
@@ -341,6 +373,18 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
     p.cvec = c.cvec;
     p.units = (uint64_t)d.outer * d.inner * p.AB * c.nchunk;
     p.nwords = (p.units + 31) / 32;
+    p.wstride = 1;
+    {
+        const uint64_t batch = (uint64_t)d.outer * d.inner;
+        const long mode = env_int("IPT_CYC_SCRAMBLE", 1);
+        if (mode && batch > 1 && p.nwords > batch && p.nwords < (1ull << 32)) {
+            uint64_t st = (p.nwords + batch - 1) / batch;
+            auto gcd = [](uint64_t a, uint64_t b) { while (b) { uint64_t t = a % b; a = b; b = t; } return a; };
+            while (gcd(st, p.nwords) != 1) ++st;
+            p.wstride = st;
+        }
+    }
+    p.divNwords = make_fastdiv(p.nwords ? p.nwords : 1);
     p.divB = make_fastdiv((uint64_t)d.B);
     p.divAB = make_fastdiv(p.AB);
     p.divInner = make_fastdiv((uint64_t)d.inner);
@@ -350,6 +394,7 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
     p.refresh = (int)env_int("IPT_CYC_REFRESH", 1);
     p.zero = 0;
     p.fence = (int)env_int("IPT_CYC_FENCE", 1);
+    p.pf = (int)env_int("IPT_CYC_PF", 0);
     cudaError_t e = cudaMemsetAsync(ws, 0, 256 + p.nwords * 4, st);
     if (e != cudaSuccess) return e;
     return fn(p, st, device);

@@ -7,21 +7,23 @@
 // 0010! stage applies it to the N'M' independent m x n tiles; BS is the fastest
 // 010! "if the tile (m x n) fits into shared memory".
 //
-// B200 design:
-//   * Fast path (elem 4/8/16 B, m and n multiples of V = 16/elem): persistent CTAs, two
-//     shared-memory tile buffers.  Each tile row (n*elem bytes, contiguous in HBM) is
-//     fetched by the TMA engine with a 1-D bulk copy (cp.async.bulk, completion on an
-//     mbarrier) into a row-padded layout; the next tile is prefetched while the current
-//     one is written out.  The padded pitch q (in 16-byte units) is odd.
-//   * Write-out: each thread owns a V x V block, reads V 16-byte row pieces from shared
-//     memory in a lane-rotated order (conflict-free: every 8-lane phase hits 8 distinct
-//     16-byte bank groups because q is odd and the row order is rotated by the lane's
-//     position), transposes the block in registers with a select-network rotation, and
-//     writes V fully coalesced 16-byte stores (a warp writes 512 contiguous bytes per
-//     output row piece).
-//   * Generic path (any elem size / any m, n that fit): one tile per iteration, plain
-//     coalesced element loads into an odd-pitch shared array, barrier, coalesced element
-//     stores from the transposed position -- Fig. 1 written for a CUDA block.
+// B200 design.  Fast paths (elem 4/8/16 B, m and n multiples of
+// V = 16/elem, 16-B aligned tiles) share the write-out and differ in how a tile reaches
+// shared memory:
+//   * "tma": persistent CTAs with an NB-deep ring of tile buffers; each tile row
+//     (n*elem contiguous bytes) is fetched by the TMA engine with a 1-D bulk copy
+//     (cp.async.bulk, completion on an mbarrier) into a row-padded layout, NB-1 tiles
+//     ahead of the one being written out.
+//   * "ldg": each thread issues a batch of 16-byte loads into registers (many bytes in
+//     flight per thread), stores them to the padded layout, barrier, write-out; several
+//     CTAs per SM overlap each other's load and store phases.
+//   Shared layout: row pitch q (16-byte units) is odd.  Write-out: each thread owns a
+//   V x V block, reads its V row pieces with a lane-rotated order (every 8-lane phase
+//   of an LDS.128 hits 8 distinct 16-byte bank groups), transposes the block in
+//   registers with a select-network rotation, and issues V coalesced 16-byte stores
+//   (a warp writes 512 contiguous bytes per output row piece).
+// Generic path (any elem size / any m, n that fit): coalesced element loads into an
+// odd-pitch shared array, barrier, coalesced element stores -- Fig. 1 for a CUDA block.
 #include "ipt_internal.h"
 #include "mem_ptx.cuh"
 
@@ -37,10 +39,11 @@ struct TileParams {
     uint64_t count;       // total tiles = outer * inner
     FastDiv divInner;
     uint32_t m, n;        // tile rows / cols (input view)
-    uint32_t q;           // fast path: padded pitch in 16-byte units (odd)
+    uint32_t q;           // fast paths: padded pitch in 16-byte units (odd)
     uint32_t pitch;       // generic path: padded pitch in elements (odd)
     uint32_t buf_bytes;   // bytes of one smem tile buffer
-    FastDiv divM, divN, divMV;  // m, n and m/V
+    uint32_t nbuf;        // tma path: ring depth
+    FastDiv divM, divN, divMV, divNV;  // m, n, m/V, n/V
 };
 
 __device__ __forceinline__ char *tile_ptr(const TileParams &p, uint64_t t) {
@@ -90,78 +93,121 @@ template <> __device__ __forceinline__ uint4 pack<8>(const unsigned long long (&
 }
 template <> __device__ __forceinline__ uint4 pack<16>(const uint4 (&e)[1]) { return e[0]; }
 
-// ---------------------------------------------------------------------- fast kernel
+__device__ __forceinline__ void sts128(uint32_t saddr, const uint4 &v) {
+    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};"
+                 :: "r"(saddr), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+
+// Write the transposed tile from padded shared memory (sbase, pitch q) to global g.
 template <int EB>
-__global__ void __launch_bounds__(256) tile_onchip_fast(const TileParams p) {
-    constexpr int V = 16 / EB;               // elements per 16-byte vector
-    constexpr int ROT = (V >= 8) ? 1 : 8 / V; // lanes sharing one rotation
+__device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, char *g) {
+    constexpr int V = 16 / EB;
+    constexpr int ROT = (V >= 8) ? 1 : 8 / V;   // lanes sharing one rotation
     using E = typename Elem<EB>::T;
+    const uint32_t nblk = (p.m / V) * (p.n / V);
+    for (uint32_t blk = threadIdx.x; blk < nblk; blk += blockDim.x) {
+        uint64_t bj64, bi64;
+        fdivmod(blk, p.divMV, bj64, bi64);
+        const uint32_t bi = (uint32_t)bi64, bj = (uint32_t)bj64;
+        const int off = (int)((bi / ROT) % V);
+        E x[V][V];
+#pragma unroll
+        for (int kk = 0; kk < V; ++kk) {
+            const uint32_t rho = (uint32_t)((kk + off) % V);
+            const uint4 v = lds128(sbase + ((bi * V + rho) * p.q + bj) * 16);
+            unpack<EB>(v, x[kk]);
+        }
+        // x[kk][c] = tile[bi*V + (kk+off)%V][bj*V + c]; output row bj*V+c gets column c.
+#pragma unroll
+        for (int c = 0; c < V; ++c) {
+            E col[V];
+#pragma unroll
+            for (int kk = 0; kk < V; ++kk) col[kk] = x[kk][c];
+            rotate_sel<V, E>(col, off);    // col[e] = tile[bi*V + e][bj*V + c]
+            stg128_na(g + ((size_t)(bj * V + c) * p.m + (size_t)bi * V) * EB, pack<EB>(col));
+        }
+    }
+}
+
+// ------------------------------------------------------------------- TMA ring kernel
+template <int EB>
+__global__ void __launch_bounds__(512) tile_onchip_tma(const TileParams p) {
     extern __shared__ __align__(128) unsigned char smem[];
-    uint64_t *bar = reinterpret_cast<uint64_t *>(smem);
+    uint64_t *bar = reinterpret_cast<uint64_t *>(smem);     // up to 8 mbarriers
     unsigned char *const buf0 = smem + 128;
     const int tid = threadIdx.x;
-    const int nthr = blockDim.x;
     const int lane = tid & 31;
-    const uint32_t mv = p.m / V, nv = p.n / V;
-    const uint32_t nblk = mv * nv;
     const uint32_t row_bytes = p.n * EB;
+    const uint32_t NB = p.nbuf;
 
     if (tid == 0) {
-        mbar_init(&bar[0], 1);
-        mbar_init(&bar[1], 1);
+        for (uint32_t b = 0; b < NB; ++b) mbar_init(&bar[b], 1);
         fence_mbar_init();
     }
     __syncthreads();
 
-    auto issue = [&](uint64_t t, int b) {
-        // warp 0 only: lane 0 arms the barrier, then all lanes issue row copies
+    auto issue = [&](uint64_t t, uint32_t b) {   // warp 0 only
         const char *g = tile_ptr(p, t);
         if (lane == 0) mbar_arrive_expect_tx(&bar[b], (uint32_t)p.tile_bytes);
         __syncwarp();
+        unsigned char *dst = buf0 + (size_t)b * p.buf_bytes;
         for (uint32_t i = lane; i < p.m; i += 32)
-            bulk_g2s(buf0 + (size_t)b * p.buf_bytes + (size_t)i * p.q * 16, g + (size_t)i * row_bytes, row_bytes, &bar[b]);
+            bulk_g2s(dst + (size_t)i * p.q * 16, g + (size_t)i * row_bytes, row_bytes, &bar[b]);
     };
 
-    uint64_t t = blockIdx.x;
-    if (t < p.count && tid < 32) issue(t, 0);
-    for (int it = 0; t < p.count; t += gridDim.x, ++it) {
-        const int b = it & 1;
-        const uint64_t tn = t + gridDim.x;
-        if (tn < p.count && tid < 32) issue(tn, b ^ 1);
-        mbar_wait(&bar[b], (uint32_t)((it >> 1) & 1));
+    // prologue: NB - 1 tiles in flight
+    if (tid < 32) {
+        for (uint32_t j = 0; j + 1 < NB; ++j) {
+            const uint64_t t = blockIdx.x + (uint64_t)j * gridDim.x;
+            if (t < p.count) issue(t, j);
+        }
+    }
+    uint32_t it = 0;
+    for (uint64_t t = blockIdx.x; t < p.count; t += gridDim.x, ++it) {
+        const uint32_t b = it % NB;
+        const uint64_t tn = t + (uint64_t)(NB - 1) * gridDim.x;
+        // buffer (it + NB - 1) % NB was consumed in iteration it - 1 (barrier below)
+        if (tn < p.count && tid < 32) issue(tn, (it + NB - 1) % NB);
+        mbar_wait(&bar[b], (it / NB) & 1);
+        write_out<EB>(p, smem_u32(buf0) + b * p.buf_bytes, tile_ptr(p, t));
+        __syncthreads();
+    }
+}
 
+// ------------------------------------------------------------ register-staged kernel
+template <int EB, int U>
+__global__ void __launch_bounds__(512) tile_onchip_ldg(const TileParams p) {
+    extern __shared__ __align__(128) unsigned char smem[];
+    const uint32_t sbase = smem_u32(smem);
+    const uint32_t nvec = (uint32_t)(p.tile_bytes / 16);
+    for (uint64_t t = blockIdx.x; t < p.count; t += gridDim.x) {
         char *g = tile_ptr(p, t);
-        const uint32_t sbase = smem_u32(buf0) + (uint32_t)b * p.buf_bytes;
-        for (uint32_t blk = tid; blk < nblk; blk += nthr) {
-            uint64_t bj64, bi64;
-            fdivmod(blk, p.divMV, bj64, bi64);
-            const uint32_t bi = (uint32_t)bi64, bj = (uint32_t)bj64;
-            const int off = (int)((bi / ROT) % V);
-            E x[V][V];
+        for (uint32_t e0 = threadIdx.x; e0 < nvec; e0 += U * blockDim.x) {
+            uint4 v[U];
 #pragma unroll
-            for (int kk = 0; kk < V; ++kk) {
-                const uint32_t rho = (uint32_t)((kk + off) % V);
-                const uint4 v = lds128(sbase + ((bi * V + rho) * p.q + bj) * 16);
-                unpack<EB>(v, x[kk]);
+            for (int u = 0; u < U; ++u) {
+                const uint32_t e = e0 + u * blockDim.x;
+                if (e < nvec) v[u] = ld_cg<16>(g + (size_t)e * 16);
             }
-            // x[kk][c] = tile[bi*V + (kk+off)%V][bj*V + c]; output row c gets column c.
 #pragma unroll
-            for (int c = 0; c < V; ++c) {
-                E col[V];
-#pragma unroll
-                for (int kk = 0; kk < V; ++kk) col[kk] = x[kk][c];
-                rotate_sel<V, E>(col, off);    // col[e] = tile[bi*V + e][bj*V + c]
-                stg128_na(g + ((size_t)(bj * V + c) * p.m + (size_t)bi * V) * EB, pack<EB>(col));
+            for (int u = 0; u < U; ++u) {
+                const uint32_t e = e0 + u * blockDim.x;
+                if (e < nvec) {
+                    uint64_t i, j;
+                    fdivmod(e, p.divNV, i, j);
+                    sts128(sbase + ((uint32_t)i * p.q + (uint32_t)j) * 16, v[u]);
+                }
             }
         }
-        __syncthreads();   // buffer b fully consumed before it is refilled (it + 2)
+        __syncthreads();
+        write_out<EB>(p, sbase, g);
+        __syncthreads();
     }
-    (void)lane;
 }
 
 // ------------------------------------------------------------------- generic kernel
 template <typename T>
-__global__ void __launch_bounds__(256) tile_onchip_generic(const TileParams p) {
+__global__ void __launch_bounds__(512) tile_onchip_generic(const TileParams p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     T *s = reinterpret_cast<T *>(smem_raw);
     const uint32_t mn = p.m * p.n;
@@ -185,39 +231,56 @@ __global__ void __launch_bounds__(256) tile_onchip_generic(const TileParams p) {
 // ------------------------------------------------------------------------ host side
 namespace {
 
-bool fast_ok(const StageDesc &d) {
-    const int eb = d.eb;
+enum { MODE_LDG = 0, MODE_TMA = 1 };
+
+int tile_mode() { return (int)env_int("IPT_TILE_MODE", MODE_LDG); }
+int tile_threads() {
+    long t = env_int("IPT_TILE_THREADS", 512);
+    return (t == 256 || t == 512) ? (int)t : 512;
+}
+uint32_t tma_nbuf() {
+    long b = env_int("IPT_TILE_STAGES", 2);
+    return (uint32_t)(b < 2 ? 2 : (b > 8 ? 8 : b));
+}
+
+bool vec_ok(int64_t A, int64_t B, int eb) {
     if (eb != 4 && eb != 8 && eb != 16) return false;
     const int V = 16 / eb;
-    if (d.A % V || d.B % V) return false;
+    if (A % V || B % V) return false;
+    return !env_int("IPT_TILE_GENERIC", 0);
+}
+
+bool fast_ok(const StageDesc &d) {
+    if (!vec_ok(d.A, d.B, d.eb)) return false;
     if (((uintptr_t)d.base & 15) != 0) return false;
     if (d.outer > 1 && (d.ostride & 15) != 0) return false;
-    if (env_int("IPT_TILE_GENERIC", 0)) return false;
     return true;
 }
 
-uint32_t fast_q(const StageDesc &d) {
-    uint32_t q = (uint32_t)(d.B * d.eb / 16);
+uint32_t fast_q(int64_t B, int eb) {
+    uint32_t q = (uint32_t)(B * eb / 16);
     return (q & 1) ? q : q + 1;
 }
 
-size_t fast_smem(const StageDesc &d) {
-    return 128 + 2 * (size_t)d.A * fast_q(d) * 16;
+size_t fast_smem(int64_t A, int64_t B, int eb) {
+    const size_t buf = (size_t)A * fast_q(B, eb) * 16;
+    if (tile_mode() == MODE_TMA) return 128 + tma_nbuf() * buf;
+    return buf;
 }
 
-uint32_t generic_pitch(const StageDesc &d) {
-    uint32_t P = (uint32_t)d.B;
+uint32_t generic_pitch(int64_t B) {
+    uint32_t P = (uint32_t)B;
     return (P & 1) ? P : P + 1;
 }
 
-size_t generic_smem(const StageDesc &d) { return (size_t)d.A * generic_pitch(d) * d.eb; }
+size_t generic_smem(int64_t A, int64_t B, int eb) { return (size_t)A * generic_pitch(B) * eb; }
 
 template <typename K>
-int occupancy(K kern, size_t smem, int device) {
+int occupancy(K kern, int threads, size_t smem, int device) {
     static std::mutex mu;
-    static std::map<std::pair<const void *, std::pair<int, size_t>>, int> cache;
+    static std::map<std::pair<const void *, std::pair<int, std::pair<int, size_t>>>, int> cache;
     std::lock_guard<std::mutex> lk(mu);
-    auto key = std::make_pair((const void *)kern, std::make_pair(device, smem));
+    auto key = std::make_pair((const void *)kern, std::make_pair(device, std::make_pair(threads, smem)));
     auto it = cache.find(key);
     if (it != cache.end()) return it->second;
     int n = 0;
@@ -225,7 +288,7 @@ int occupancy(K kern, size_t smem, int device) {
     // shape would make a later, larger launch fail)
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          dev_props(device).smem_optin);
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, 256, smem) != cudaSuccess) n = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, threads, smem) != cudaSuccess) n = 1;
     if (n < 1) n = 1;
     cache[key] = n;
     return n;
@@ -234,11 +297,12 @@ int occupancy(K kern, size_t smem, int device) {
 template <typename K>
 cudaError_t go(K kern, const TileParams &p, size_t smem, cudaStream_t st, int device) {
     DevProps dp = dev_props(device);
-    int per_sm = occupancy(kern, smem, device);
+    const int threads = tile_threads();
+    int per_sm = occupancy(kern, threads, smem, device);
     uint64_t grid = (uint64_t)dp.sms * per_sm;
     if (p.count < grid) grid = p.count;
     if (grid < 1) grid = 1;
-    kern<<<(unsigned)grid, 256, smem, st>>>(p);
+    kern<<<(unsigned)grid, threads, smem, st>>>(p);
     note_launch();
     return cudaGetLastError();
 }
@@ -247,14 +311,9 @@ cudaError_t go(K kern, const TileParams &p, size_t smem, cudaStream_t st, int de
 
 int tile_onchip_path(int64_t A, int64_t B, int eb, int device) {
     DevProps dp = dev_props(device);
-    StageDesc d{};
-    d.A = A; d.B = B; d.s = 1; d.eb = eb; d.outer = 1; d.inner = 1;
-    d.base = nullptr;
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
-    const bool vec = (eb == 4 || eb == 8 || eb == 16) && A % (16 / eb) == 0 && B % (16 / eb) == 0
-                     && !env_int("IPT_TILE_GENERIC", 0);
-    if (vec && (long)fast_smem(d) <= budget) return 2;
-    if ((long)generic_smem(d) <= budget && A * B < (1ll << 31)) return 1;
+    if (vec_ok(A, B, eb) && (long)fast_smem(A, B, eb) <= budget) return 2;
+    if ((long)generic_smem(A, B, eb) <= budget && A * B < (1ll << 31)) return 1;
     return 0;
 }
 
@@ -275,19 +334,30 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
     p.divM = make_fastdiv((uint64_t)d.A);
     p.divN = make_fastdiv((uint64_t)d.B);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
-    if (fast_ok(d) && (long)fast_smem(d) <= budget) {
-        p.q = fast_q(d);
+    if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) <= budget) {
+        const int V = 16 / d.eb;
+        p.q = fast_q(d.B, d.eb);
         p.buf_bytes = (uint32_t)((size_t)d.A * p.q * 16);
-        p.divMV = make_fastdiv((uint64_t)(d.A / (16 / d.eb)));
-        const size_t smem = fast_smem(d);
-        switch (d.eb) {
-            case 4: return go(tile_onchip_fast<4>, p, smem, st, device);
-            case 8: return go(tile_onchip_fast<8>, p, smem, st, device);
-            case 16: return go(tile_onchip_fast<16>, p, smem, st, device);
+        p.divMV = make_fastdiv((uint64_t)(d.A / V));
+        p.divNV = make_fastdiv((uint64_t)(d.B / V));
+        p.nbuf = tma_nbuf();
+        const size_t smem = fast_smem(d.A, d.B, d.eb);
+        if (tile_mode() == MODE_TMA) {
+            switch (d.eb) {
+                case 4: return go(tile_onchip_tma<4>, p, smem, st, device);
+                case 8: return go(tile_onchip_tma<8>, p, smem, st, device);
+                case 16: return go(tile_onchip_tma<16>, p, smem, st, device);
+            }
+        } else {
+            switch (d.eb) {
+                case 4: return go(tile_onchip_ldg<4, 8>, p, smem, st, device);
+                case 8: return go(tile_onchip_ldg<8, 8>, p, smem, st, device);
+                case 16: return go(tile_onchip_ldg<16, 8>, p, smem, st, device);
+            }
         }
     }
-    p.pitch = generic_pitch(d);
-    const size_t smem = generic_smem(d);
+    p.pitch = generic_pitch(d.B);
+    const size_t smem = generic_smem(d.A, d.B, d.eb);
     if ((long)smem > budget) return cudaErrorInvalidValue;
     switch (d.eb) {
         case 1: return go(tile_onchip_generic<uint8_t>, p, smem, st, device);

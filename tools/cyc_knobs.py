@@ -1,0 +1,28 @@
+"""cycle_global throughput for a few super-element sizes under knob settings (env)."""
+import os, sys, json, itertools
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import paper_conf_ppopp_sunggggh14_b200 as ipt
+dev = torch.device("cuda", 0)
+TOT = 12800 * 15000
+buf = torch.empty(TOT, dtype=torch.int32, device=dev)
+buf.random_()
+def bench(batch, A, B, s, reps=3):
+    ipt.ipt_100_(buf, batch, A, B, s); ipt.ipt_100_(buf, batch, B, A, s)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for r in range(reps):
+        ipt.ipt_100_(buf, batch, A, B, s); ipt.ipt_100_(buf, batch, B, A, s)
+    e1.record(); torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / (2 * reps)
+    return round(2 * batch * A * B * s * 4 / (ms / 1e3) / 1e9)
+knobs = [dict(IPT_CYC_SCRAMBLE="0"), dict(), dict(IPT_CYC_FENCE="0"),
+         dict(IPT_CYC_G="8", IPT_CYC_R="4"), dict(IPT_CYC_G="8", IPT_CYC_R="4", IPT_CYC_FENCE="0")]
+for kn in knobs:
+    for k in list(os.environ):
+        if k.startswith("IPT_CYC"): del os.environ[k]
+    os.environ.update(kn)
+    res = {"S512_st1": bench(1, 12800, 15000 // 128, 128), "S512_st3": bench(75, 100, 200, 128),
+           "S320_st3": bench(75, 160, 200, 80), "S800_st3": bench(75, 64, 200, 200), "S240_st1": bench(1, 12800, 250, 60)}
+    print(json.dumps(kn), json.dumps(res), flush=True)

@@ -1,0 +1,30 @@
+"""Microbenchmark of the tile stage (0010!) alone across modes / tile shapes."""
+import os, sys, itertools, json
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import paper_conf_ppopp_sunggggh14_b200 as ipt
+dev = torch.device("cuda", 0)
+TOT = 12800 * 15000  # elements (768 MB f32)
+buf = torch.empty(TOT, dtype=torch.int32, device=dev)
+buf.random_()
+def bench(m, n, reps=5):
+    cnt = TOT // (m * n)
+    ipt.ipt_010_(buf, cnt, m, n); ipt.ipt_010_(buf, cnt, n, m)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for r in range(reps):
+        ipt.ipt_010_(buf, cnt, m, n); ipt.ipt_010_(buf, cnt, n, m)
+    e1.record(); torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / (2 * reps)
+    return 2 * cnt * m * n * 4 / (ms / 1e3) / 1e9
+shapes = [(128, 200), (160, 160), (200, 128), (100, 100), (64, 200), (80, 80), (60, 60), (128, 128), (32, 256), (48, 48)]
+for mode, thr, st in [("0", "512", "2"), ("0", "256", "2"), ("1", "256", "2"), ("1", "512", "2"), ("1", "512", "3"), ("1", "512", "4")]:
+    os.environ["IPT_TILE_MODE"] = mode; os.environ["IPT_TILE_THREADS"] = thr; os.environ["IPT_TILE_STAGES"] = st
+    res = {}
+    for (m, n) in shapes:
+        try:
+            res[f"{m}x{n}"] = round(bench(m, n), 0)
+        except Exception as e:
+            res[f"{m}x{n}"] = str(e)[:40]
+    print(f"mode={'ldg' if mode=='0' else 'tma'} threads={thr} stages={st}", json.dumps(res), flush=True)

@@ -60,18 +60,13 @@ def fill_device_(buf, M: int, N: int, elem_bytes: int, t0: int = 0, count: int =
 
     n = count * M * N
     assert buf.numel() >= n
-    lin = torch.arange(t0 * M * N, t0 * M * N + n, device=buf.device, dtype=torch.int64)
-    if elem_bytes == 8:
-        # uint64 wrap-around arithmetic on int64 two's complement is identical bitwise.
-        mul = _MUL64 - (1 << 64)
-        v = lin * mul + seed
-        buf[:n].copy_(v.view(buf.dtype) if buf.dtype == torch.int64 else v)
-    elif elem_bytes == 4:
-        v = (lin * _MUL32 + seed) & 0xFFFFFFFF
-        v = torch.where(v >= 2 ** 31, v - 2 ** 32, v).to(torch.int32)
-        buf[:n].copy_(v)
-    else:
+    if elem_bytes not in (4, 8):
         raise ValueError("device fill supports 4- and 8-byte elements")
+    CH = 1 << 27   # bounded temporaries
+    for c0 in range(0, n, CH):
+        c1 = min(n, c0 + CH)
+        lin = torch.arange(t0 * M * N + c0, t0 * M * N + c1, device=buf.device, dtype=torch.int64)
+        buf[c0:c1].copy_(values_torch_sample(lin, elem_bytes, seed))
     return buf
 
 

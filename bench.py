@@ -283,6 +283,7 @@ def main():
     kern_bytes = {"cycle_global": 0, "tile_onchip": 0}
     kern_n = {"cycle_global": 0, "tile_onchip": 0}
     stage_scaled = None
+    per_shape = {}
     if "batch" not in wl:
         orient_sim = list(orient_before)
         S_bytes = 0
@@ -290,6 +291,7 @@ def main():
             for i, (t, M, N, cnt, _) in enumerate(mats):
                 a, b = (N, M) if orient_sim[i] else (M, N)
                 p = plans[(a, b)]
+                ps = per_shape.setdefault(f"{a}x{b}", {"ms": 0.0, "n": 0, "stage_ms": [0.0, 0.0, 0.0]})
                 for st in range(3):
                     v = ipt.VARIANTS[p.variant[st]]
                     if v == "identity":
@@ -299,7 +301,16 @@ def main():
                     kern_bytes[v] += 2 * a * b * eb
                     kern_n[v] += 1
                     S_bytes += 2 * a * b * eb
+                    ps["ms"] += dt
+                    ps["stage_ms"][st] += dt
+                ps["n"] += 1
                 orient_sim[i] = not orient_sim[i]
+        for key, ps in per_shape.items():
+            a, b = (int(x) for x in key.split("x"))
+            ps["eff_gbs"] = round(2 * a * b * eb * ps["n"] / (ps["ms"] / 1e3) / 1e9, 1)
+            ps["stage_gbs"] = [round(2 * a * b * eb * ps["n"] / (x / 1e3) / 1e9, 1) if x else None
+                               for x in ps["stage_ms"]]
+            del ps["ms"], ps["stage_ms"]
         stage_scaled = (S_bytes / (elapsed_ms / 1e3) / 1e9) / peak
     dom = max(kern_t, key=lambda k: kern_t[k]) if any(kern_t.values()) else None
     roofline = None
@@ -411,7 +422,7 @@ def main():
                        "l2": "no flush: every matrix exceeds the 126 MB L2" if args.workload in ("sweep", "c3", "c4", "c5") else "L2-resident (52 MB)",
                        "parallelism": f"replicas x{world}" if "batch" not in wl else f"batch shards x{world}"},
             "hbm_frac_stage_scaled": round(stage_scaled, 4) if stage_scaled else None,
-            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
+            "per_shape": per_shape, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
             "clocks": clk, "verified": ok,
         }
         print(json.dumps(line), flush=True)

@@ -96,6 +96,8 @@ def lib():
             f.argtypes = args
         L.ipt__fastdiv.restype = ctypes.c_uint64
         L.ipt__fastdiv.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
+        L.ipt__fastdiv32.restype = ctypes.c_uint32
+        L.ipt__fastdiv32.argtypes = [ctypes.c_uint32, ctypes.c_uint32]
         _lib = L
     return _lib
 

@@ -13,28 +13,46 @@
 //   * A "walker" is a group of G lanes (G | 32) holding one super-element (or one chunk
 //     of it) in registers as W-byte vectors (W = 16 when alignment permits), R vectors per
 //     lane.  A warp runs 32/G walkers in lock-step, so a warp keeps 32/G independent
-//     chains in flight (Little's law); a persistent grid fills every SM.
+//     chains in flight (Little's law); a persistent grid fills every SM.  With G = 32 all
+//     control flow is warp-uniform.
 //   * Super-elements larger than one walker's capacity are split into `nchunk` chunks
 //     that follow the SAME permutation independently (moving chunk c of every
 //     super-element is itself a valid permutation), each with its own flag bit.
-//   * Start positions are handed out in increasing order, 32 units (one flag word) at a
-//     time, from a global work counter (adjacent work-items start at adjacent
-//     elements); the flag word doubles as a pre-check so claimed units are never
-//     re-read.
-//   * Claim protocol (P1): flag bit u = "unit u has received its final
-//     value".  Chain step from cur: d = next(cur); load backup = A[d] and atomicOr(bit d)
-//     concurrently; if the bit was already set the chain ends, else store carried data
-//     into d and carry the backup on.  A chain start at x loads A[x] and then re-checks
-//     bit x with a load whose address depends on the loaded data (so it is ordered after
-//     it); if set, the start is abandoned (the claimer of x carries A[x]).
-//   * Index maps use 64-bit indices and multiply-high division (no 64-bit '%').
+//   * Start units are handed out 32 at a time (one flag word, which doubles as a
+//     pre-check so claimed units are never re-read) from a global work counter: in
+//     increasing order for one matrix (adjacent work-items start at adjacent elements,
+//     P:172), scrambled across a batch so that all matrices' start frontiers advance
+//     together (fewer, longer chains).
+//   * Claim protocol (P1; modelled in tools/protocol_sim.py): flag bit u =
+//     "unit u has received its final value".  Chain step from cur: d = next(cur); load
+//     backup = A[d] and claim bit d (atomic OR, acquire) concurrently; a lost claim ends
+//     the chain, a won claim stores the carried data into d (after the claim) and carries
+//     the backup on.  A cycle that closes at the walker's own start is claimed like any
+//     other target (its backup is not re-read).  A chain start at x loads A[x], fences,
+//     and re-checks bit x; if set, the start is abandoned (the claimer of x carries A[x]).
+//   * Index maps use multiply-high division (no '%' or '/' in the loop), in 32-bit
+//     arithmetic whenever every index fits (I = uint32_t), else 64-bit.
 #include "ipt_internal.h"
 #include "mem_ptx.cuh"
 
-#include <mutex>
 #include <map>
+#include <mutex>
 
 namespace ipt {
+
+__device__ __forceinline__ void fdivmod_t(uint32_t n, const FastDiv32 &f, const FastDiv &,
+                                          uint32_t &q, uint32_t &r) {
+    fdivmod32(n, f, q, r);
+}
+__device__ __forceinline__ void fdivmod_t(uint64_t n, const FastDiv32 &, const FastDiv &f,
+                                          uint64_t &q, uint64_t &r) {
+    fdivmod(n, f, q, r);
+}
+
+struct Div2 {
+    FastDiv d64;
+    FastDiv32 d32;
+};
 
 struct CycParams {
     char *base;
@@ -47,35 +65,45 @@ struct CycParams {
     uint64_t nvec;      // vectors per super-element
     uint64_t units;     // batch * A*B * nchunk
     uint64_t nwords;    // flag words
-    FastDiv divB, divAB, divInner, divNchunk;
+    uint64_t wstride;   // start-order scramble (coprime to nwords)
+    Div2 divB, divAB, divInner, divNchunk, divNwords;
     uint32_t *flags;
     unsigned long long *counter;
     int refresh;        // re-read the flag word after a chain ends before the next start
-    uint32_t zero;      // always 0 at run time; opaque to the compiler (see dep_zero use)
     int fence;          // 1: PTX-model fences on both sides of the claim protocol
-    int pf;             // chain look-ahead depth (L2 prefetch of the next targets)
-    uint64_t wstride;   // start-order scramble (coprime to nwords)
-    FastDiv divNwords;
+    uint32_t zero;      // 0 at run time, opaque to the compiler (address-dependency knob)
+    unsigned long long *stats;  // optional diagnostics (IPT_CYC_STATS=1): round counts
+    int debug;          // diagnostics only (IPT_CYC_DEBUG), never set by the library
 };
 
 enum : int { M_FETCH = 0, M_SCAN = 1, M_START = 2, M_CHAIN = 3, M_REFRESH = 4, M_DONE = 5 };
 
-template <int W, int G, int R>
-__global__ void __launch_bounds__(256) cycle_global_kernel(const CycParams p) {
+// Register budget -> resident warps: the kernel is latency-bound (one dependent round
+// trip per chain step), so it is compiled for full occupancy (8 x 256 threads = 64 warps
+// per SM, <= 32 registers) when a walker's payload is <= 16 bytes per lane.
+template <int W, int R> struct CycMinBlocks {
+    static constexpr int value = (W * R <= 16) ? 8 : ((W * R <= 32) ? 6 : 4);
+};
+
+template <int W, int G, int R, typename I>
+__global__ void __launch_bounds__(256, CycMinBlocks<W, R>::value)
+cycle_global_kernel(const CycParams p) {
     using V = typename VecT<W>::type;
     constexpr unsigned FULL = 0xffffffffu;
     const int lane = threadIdx.x & 31;
     const int gl = lane % G;          // lane within walker group
     const int g0 = lane - gl;         // first lane of the group
     const unsigned gmask = (G == 32) ? FULL : (((1u << G) - 1u) << g0);
+    const I A = (I)p.A, nchunk = (I)p.nchunk, nwords = (I)p.nwords;
 
     int mode = M_FETCH;
-    uint64_t word = 0;     // flag word (= chunk of 32 start units) being scanned
+    uint32_t st_start = 0, st_abort = 0, st_step = 0, st_lost = 0, st_refresh = 0, st_iter = 0;
+    I word = 0;            // flag word (= 32 start units) being scanned
     uint32_t cw = 0;       // cached copy of that flag word
     int nb = 0;            // next bit to consider in the word
     char *item = nullptr;  // start of the current batch item (+ chunk offset)
-    uint64_t ubase = 0;    // unit index of (item, k = 0, chunk)
-    uint64_t k = 0, k0 = 0;
+    I ubase = 0;           // unit index of (item, k = 0, chunk)
+    I k = 0, k0 = 0;
     int nv = 0;            // vectors in this chunk
     V data[R], in[R];
 #pragma unroll
@@ -90,17 +118,13 @@ __global__ void __launch_bounds__(256) cycle_global_kernel(const CycParams p) {
                 unsigned long long wb = 0;
                 if (lane == leader) wb = atomicAdd(p.counter, (unsigned long long)__popc(need));
                 wb = __shfl_sync(FULL, wb, leader);
-                uint64_t mine = wb + __popc(need & ((1u << g0) - 1u));
-                const bool have = mine < p.nwords;
-                // Start order: fetch i scans flag word (i * wstride) mod nwords.  For a
-                // batch of small independent matrices wstride ~ words per matrix, so the
-                // start frontier advances through all matrices at once (like one big
-                // matrix) instead of bursting through one at a time, which keeps chains
-                // long and PTTWAC's redundant start reads low.
+                uint64_t mine64 = wb + __popc(need & ((1u << g0) - 1u));
+                const bool have = mine64 < p.nwords;
+                I mine = (I)mine64;
                 if (have && p.wstride != 1) {
                     uint64_t q, r;
-                    fdivmod(mine * p.wstride, p.divNwords, q, r);
-                    mine = r;
+                    fdivmod(mine64 * p.wstride, p.divNwords.d64, q, r);
+                    mine = (I)r;
                 }
                 uint32_t fw = 0;
                 if (mode == M_FETCH && have) fw = ld_relaxed_u32(p.flags + mine);
@@ -119,46 +143,55 @@ __global__ void __launch_bounds__(256) cycle_global_kernel(const CycParams p) {
             // Scan the cached word for the next unit that still needs a start walker.
             while (mode == M_SCAN) {
                 uint32_t valid = 0xffffffffu;
-                if (word == p.nwords - 1 && (p.units & 31)) valid = (1u << (p.units & 31)) - 1u;
+                if (word == nwords - 1 && (p.units & 31)) valid = (1u << (p.units & 31)) - 1u;
                 const uint32_t cand = ~cw & valid & (nb >= 32 ? 0u : (0xffffffffu << nb));
                 if (!cand) { mode = M_FETCH; break; }
                 const int b = __ffs(cand) - 1;
                 nb = b + 1;
-                const uint64_t u = word * 32 + (uint64_t)b;
-                uint64_t tk = u, ch = 0;
-                if (p.nchunk > 1) fdivmod(u, p.divNchunk, tk, ch);
-                uint64_t T, kk;
-                fdivmod(tk, p.divAB, T, kk);
-                uint64_t q, r;
-                fdivmod(kk, p.divB, q, r);
-                if (r * p.A + q == kk) continue;        // fixed point of Eq. (1): nothing moves
-                uint64_t to, ti;
-                fdivmod(T, p.divInner, to, ti);
-                item = p.base + to * p.ostride + ti * p.istride + ch * p.cvec * W;
-                ubase = T * p.AB * p.nchunk + ch;
-                nv = (int)((ch == p.nchunk - 1) ? (p.nvec - ch * p.cvec) : p.cvec);
+                const I u = word * 32 + (I)b;
+                I tk = u, ch = 0;
+                if (p.nchunk > 1) fdivmod_t(u, p.divNchunk.d32, p.divNchunk.d64, tk, ch);
+                I T, kk, q, r;
+                fdivmod_t(tk, p.divAB.d32, p.divAB.d64, T, kk);
+                fdivmod_t(kk, p.divB.d32, p.divB.d64, q, r);
+                if (r * A + q == kk) continue;          // fixed point of Eq. (1): nothing moves
+                I to, ti;
+                fdivmod_t(T, p.divInner.d32, p.divInner.d64, to, ti);
+                item = p.base + (uint64_t)to * p.ostride + (uint64_t)ti * p.istride +
+                       (uint64_t)ch * p.cvec * W;
+                ubase = T * (I)p.AB * nchunk + ch;
+                nv = (int)((ch == nchunk - 1) ? (p.nvec - (uint64_t)ch * p.cvec) : p.cvec);
                 k = k0 = kk;
                 mode = M_START;
             }
             const unsigned pending = __ballot_sync(FULL, mode == M_FETCH || mode == M_SCAN);
             if (!pending) break;
         }
-        if (!__ballot_sync(FULL, mode != M_DONE)) break;
+        if (!__ballot_sync(FULL, mode != M_DONE)) {
+            if (p.stats && gl == 0) {
+                atomicAdd(p.stats + 0, (unsigned long long)st_start);
+                atomicAdd(p.stats + 1, (unsigned long long)st_abort);
+                atomicAdd(p.stats + 2, (unsigned long long)st_step);
+                atomicAdd(p.stats + 3, (unsigned long long)st_lost);
+                atomicAdd(p.stats + 4, (unsigned long long)st_refresh);
+                if (lane == 0) atomicAdd(p.stats + 5, (unsigned long long)st_iter);
+            }
+            break;
+        }
+        ++st_iter;
 
         // --------------------------------------------------------------- memory round
-        uint64_t tgt = k;
+        I tgt = k;
         if (mode == M_CHAIN) {
-            uint64_t q, r;
-            fdivmod(k, p.divB, q, r);
-            tgt = r * p.A + q;                         // Eq. (1) on super-element offsets
+            I q, r;
+            fdivmod_t(k, p.divB.d32, p.divB.d64, q, r);
+            tgt = r * A + q;                           // Eq. (1) on super-element offsets
         }
-        // Cycle closed at our own start x: x must still be CLAIMED (another walker carrying
-        // A[prev(x)] -- the start walker of prev(x) -- may race for it), but its backup is
-        // the value this walker already delivered, so it is not re-read.
         const bool back_home = (mode == M_CHAIN) && (tgt == k0);
-        const uint64_t ut = ubase + tgt * p.nchunk;    // flag index of the target unit
-        const uint32_t bit = 1u << (ut & 31);
-        char *addr = item + tgt * p.S;
+        const I ut = ubase + tgt * nchunk;             // flag index of the target unit
+        const uint32_t bit = 1u << ((uint32_t)ut & 31);
+        uint32_t *fwp = p.flags + (ut >> 5);
+        char *addr = item + (uint64_t)tgt * p.S;
 
         if ((mode == M_START || mode == M_CHAIN) && !back_home) {
 #pragma unroll
@@ -166,51 +199,59 @@ __global__ void __launch_bounds__(256) cycle_global_kernel(const CycParams p) {
                 const int v = gl + r * G;
                 if (v < nv) in[r] = ld_cg<W>(addr + (size_t)v * W);
             }
-            // Look-ahead: the chain's next positions are known from Eq. (1) alone, so the
-            // lines of the next `pf` targets are prefetched into L2 now; their backup reads
-            // (issued in later rounds, only by whoever claims them) then hit L2 instead of
-            // paying a DRAM round trip per chain step.  No data is consumed early, so the
-            // claim protocol is unchanged; a prefetch is wasted only at a chain's true end
-            // (the winner of a lost claim walks the same targets).
-            uint64_t la = tgt;
-            for (int j = 0; j < p.pf; ++j) {
-                uint64_t q, r;
-                fdivmod(la, p.divB, q, r);
-                la = r * p.A + q;
-                if (la == k0) break;
-                const uintptr_t lo = (uintptr_t)(item + la * p.S);
-                const uintptr_t first = lo & ~(uintptr_t)127;
-                const uintptr_t last = (lo + (uintptr_t)nv * W - 1) & ~(uintptr_t)127;
-                for (uintptr_t line = first + (uintptr_t)gl * 128; line <= last; line += (uintptr_t)G * 128)
-                    prefetch_l2((const void *)line);
-            }
         }
         uint32_t old = 0;
-        if (mode == M_CHAIN && gl == 0)
-            old = p.fence ? atom_or_acq_u32(p.flags + (ut >> 5), bit)
-                          : atom_or_u32(p.flags + (ut >> 5), bit);
+        if (mode == M_CHAIN && gl == 0) {
+            if (p.debug == 1) {          // DIAGNOSTIC ONLY (wrong results): non-atomic claim
+                old = ld_relaxed_u32(fwp);
+                if (!(old & bit)) *(volatile uint32_t *)fwp = old | bit;
+            } else {
+                old = p.fence ? atom_or_acq_u32(fwp, bit) : atom_or_u32(fwp, bit);
+            }
+        }
         uint32_t fw = 0;
         if (mode == M_START) {
-            if (p.fence) fence_acq_rel_gpu();
-            uint32_t acc = 0;
+            if (p.fence) {
+                fence_acq_rel_gpu();
+            } else {   // address dependency on the loaded data instead of a fence
+                uint32_t acc = 0;
 #pragma unroll
-            for (int r = 0; r < R; ++r) {
-                const int v = gl + r * G;
-                if (v < nv) acc |= fold(in[r]);
+                for (int r = 0; r < R; ++r) {
+                    const int v = gl + r * G;
+                    if (v < nv) acc |= fold(in[r]);
+                }
+                fwp += (acc & p.zero);
             }
-            fw = ld_relaxed_u32(p.flags + (ut >> 5) + (acc & p.zero));
+            fw = ld_relaxed_u32(fwp);
         } else if (mode == M_REFRESH) {
             fw = ld_relaxed_u32(p.flags + word);
         }
 
         // ------------------------------------------------------------------- resolve
-        old = __shfl_sync(FULL, old, g0);
-        __syncwarp();   // orders lane 0's (acquire) claim before the other lanes' stores
-        const unsigned seen = __ballot_sync(FULL, mode == M_START && (fw & bit));
-        const uint32_t fw0 = __shfl_sync(FULL, fw, g0);
+        uint32_t fw0;
+        bool start_lost;
+        if (G == 32) {
+            old = __shfl_sync(FULL, old, 0);
+            __syncwarp();   // orders lane 0's (acquire) claim before the other lanes' stores
+            start_lost = __any_sync(FULL, (fw & bit) != 0);
+            fw0 = fw;
+        } else {
+            old = __shfl_sync(FULL, old, g0);
+            __syncwarp();
+            const unsigned seen = __ballot_sync(FULL, mode == M_START && (fw & bit));
+            start_lost = (seen & gmask) != 0;
+            fw0 = __shfl_sync(FULL, fw, g0);
+        }
+        if (p.stats) {
+            st_start += (mode == M_START);
+            st_abort += (mode == M_START && start_lost);
+            st_step += (mode == M_CHAIN && !(old & bit));
+            st_lost += (mode == M_CHAIN && (old & bit));
+            st_refresh += (mode == M_REFRESH);
+        }
         if (mode == M_START) {
             cw |= fw0;
-            if (seen & gmask) {
+            if (start_lost) {
                 mode = M_SCAN;                         // already claimed: its claimer carries A[x]
             } else {
 #pragma unroll
@@ -290,9 +331,9 @@ Choice choose(const StageDesc &d) {
     return c;
 }
 
-template <int W, int G, int R>
+template <int W, int G, int R, typename I>
 cudaError_t launch_t(const CycParams &p, cudaStream_t st, int device) {
-    auto kern = cycle_global_kernel<W, G, R>;
+    auto kern = cycle_global_kernel<W, G, R, I>;
     static std::mutex mu;
     static std::map<int, int> occ_cache;
     int per_sm = 0;
@@ -322,10 +363,15 @@ cudaError_t launch_t(const CycParams &p, cudaStream_t st, int device) {
 
 typedef cudaError_t (*LaunchFn)(const CycParams &, cudaStream_t, int);
 
-#define IPT_CASE(W_, G_, R_) \
-    if (c.W == W_ && c.G == G_ && c.R == R_) return &launch_t<W_, G_, R_>;
+template <int W, int G, int R>
+LaunchFn pick_idx(bool idx32) {
+    return idx32 ? &launch_t<W, G, R, uint32_t> : &launch_t<W, G, R, uint64_t>;
+}
 
-LaunchFn lookup(const Choice &c) {
+#define IPT_CASE(W_, G_, R_) \
+    if (c.W == W_ && c.G == G_ && c.R == R_) return pick_idx<W_, G_, R_>(idx32);
+
+LaunchFn lookup(const Choice &c, bool idx32) {
     // W = 16: every group width
     IPT_CASE(16, 1, 1) IPT_CASE(16, 2, 1) IPT_CASE(16, 4, 1) IPT_CASE(16, 8, 1)
     IPT_CASE(16, 16, 1) IPT_CASE(16, 32, 1) IPT_CASE(16, 32, 2) IPT_CASE(16, 32, 4)
@@ -341,12 +387,17 @@ LaunchFn lookup(const Choice &c) {
 }
 #undef IPT_CASE
 
+Div2 make_div2(uint64_t d) {
+    Div2 x;
+    x.d64 = make_fastdiv(d);
+    x.d32 = make_fastdiv32((uint32_t)(d < (1ull << 32) ? d : 1));
+    return x;
+}
+
 }  // namespace
 
 size_t cycle_ws_bytes(const StageDesc &d) {
-    const uint64_t S = (uint64_t)d.s * d.eb;
     Choice c = choose(d);
-    (void)S;
     const uint64_t units = (uint64_t)d.outer * d.inner * d.A * d.B * c.nchunk;
     const uint64_t nwords = (units + 31) / 32;
     return 256 + nwords * 4;
@@ -354,11 +405,14 @@ size_t cycle_ws_bytes(const StageDesc &d) {
 
 cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, int device) {
     Choice c = choose(d);
-    LaunchFn fn = lookup(c);
+    const uint64_t units = (uint64_t)d.outer * d.inner * d.A * d.B * c.nchunk;
+    // 32-bit indices when every unit index (and word * 32 + 31) fits
+    const bool idx32 = units + 64 < (1ull << 32) && !env_int("IPT_CYC_IDX64", 0);
+    LaunchFn fn = lookup(c, idx32);
     if (!fn) {  // unsupported forced shape: fall back to the widest generic walker
         c.G = 32; c.R = 4;
         if ((uint64_t)c.G * c.R < c.cvec) return cudaErrorInvalidValue;
-        fn = lookup(c);
+        fn = lookup(c, idx32);
         if (!fn) return cudaErrorInvalidValue;
     }
     CycParams p;
@@ -371,30 +425,36 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
     p.nvec = p.S / c.W;
     p.nchunk = c.nchunk;
     p.cvec = c.cvec;
-    p.units = (uint64_t)d.outer * d.inner * p.AB * c.nchunk;
+    p.units = units;
     p.nwords = (p.units + 31) / 32;
     p.wstride = 1;
     {
         const uint64_t batch = (uint64_t)d.outer * d.inner;
-        const long mode = env_int("IPT_CYC_SCRAMBLE", 1);
+        const long mode = env_int("IPT_CYC_SCRAMBLE", 2);
+        auto gcd = [](uint64_t a, uint64_t b) { while (b) { uint64_t t = a % b; a = b; b = t; } return a; };
         if (mode && batch > 1 && p.nwords > batch && p.nwords < (1ull << 32)) {
-            uint64_t st = (p.nwords + batch - 1) / batch;
-            auto gcd = [](uint64_t a, uint64_t b) { while (b) { uint64_t t = a % b; a = b; b = t; } return a; };
-            while (gcd(st, p.nwords) != 1) ++st;
-            p.wstride = st;
+            uint64_t s = (p.nwords + batch - 1) / batch;
+            while (gcd(s, p.nwords) != 1) ++s;
+            p.wstride = s;
+        } else if (mode == 2 && p.nwords > 64 && p.nwords < (1ull << 32)) {
+            // single matrix: golden-ratio stride spreads concurrently started chains
+            uint64_t s = (uint64_t)(0.6180339887 * (double)p.nwords);
+            while (gcd(s, p.nwords) != 1) ++s;
+            p.wstride = s;
         }
     }
-    p.divNwords = make_fastdiv(p.nwords ? p.nwords : 1);
-    p.divB = make_fastdiv((uint64_t)d.B);
-    p.divAB = make_fastdiv(p.AB);
-    p.divInner = make_fastdiv((uint64_t)d.inner);
-    p.divNchunk = make_fastdiv(c.nchunk);
+    p.divNwords = make_div2(p.nwords ? p.nwords : 1);
+    p.divB = make_div2((uint64_t)d.B);
+    p.divAB = make_div2(p.AB);
+    p.divInner = make_div2((uint64_t)d.inner);
+    p.divNchunk = make_div2(c.nchunk);
     p.counter = (unsigned long long *)ws;
     p.flags = (uint32_t *)((char *)ws + 256);
     p.refresh = (int)env_int("IPT_CYC_REFRESH", 1);
-    p.zero = 0;
     p.fence = (int)env_int("IPT_CYC_FENCE", 1);
-    p.pf = (int)env_int("IPT_CYC_PF", 0);
+    p.zero = 0;
+    p.debug = (int)env_int("IPT_CYC_DEBUG", 0);
+    p.stats = env_int("IPT_CYC_STATS", 0) ? (unsigned long long *)ws + 8 : nullptr;
     cudaError_t e = cudaMemsetAsync(ws, 0, 256 + p.nwords * 4, st);
     if (e != cudaSuccess) return e;
     return fn(p, st, device);

@@ -47,6 +47,19 @@ FastDiv make_fastdiv(uint64_t d) {
     return f;
 }
 
+FastDiv32 make_fastdiv32(uint32_t d) {
+    FastDiv32 f{};
+    if (d == 0) d = 1;
+    f.d = d;
+    uint32_t l = 0;
+    if (d > 1) l = 32 - (uint32_t)__builtin_clz(d - 1);
+    const uint64_t two_l = (uint64_t)1 << l;
+    f.m = (uint32_t)((((two_l - d) << 32) / d) + 1);
+    f.s1 = l ? 1 : 0;
+    f.s2 = l ? l - 1 : 0;
+    return f;
+}
+
 DevProps dev_props(int device) {
     static std::mutex mu;
     static std::map<int, DevProps> cache;
@@ -535,5 +548,11 @@ const char *ipt_version(void) { return "libipt 0.1 (sm_100a)"; }
 // Internal self-test hook (not in the ABI): the multiply-high division used by every
 // kernel's index map, evaluated on the host.
 uint64_t ipt__fastdiv(uint64_t n, uint64_t d) { return fdiv(n, make_fastdiv(d)); }
+
+uint32_t ipt__fastdiv32(uint32_t n, uint32_t d) {
+    FastDiv32 f = make_fastdiv32(d);
+    const uint32_t t = (uint32_t)(((uint64_t)n * f.m) >> 32);
+    return (t + ((n - t) >> f.s1)) >> f.s2;
+}
 
 }  // extern "C"

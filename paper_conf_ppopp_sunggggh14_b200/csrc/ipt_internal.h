@@ -44,6 +44,24 @@ __host__ __device__ __forceinline__ void fdivmod(uint64_t n, const FastDiv &f, u
     r = n - q * f.d;
 }
 
+// 32-bit variant (same algorithm, N = 32), for indices known to fit 32 bits.
+struct FastDiv32 {
+    uint32_t d, m, s1, s2;
+};
+
+FastDiv32 make_fastdiv32(uint32_t d);  // host
+
+__host__ __device__ __forceinline__ void fdivmod32(uint32_t n, const FastDiv32 &f, uint32_t &q,
+                                          uint32_t &r) {
+#if defined(__CUDA_ARCH__)
+    const uint32_t t = __umulhi(n, f.m);
+#else
+    const uint32_t t = (uint32_t)(((uint64_t)n * f.m) >> 32);
+#endif
+    q = (t + ((n - t) >> f.s1)) >> f.s2;
+    r = n - q * f.d;
+}
+
 // ------------------------------------------------------------------ stage descriptor
 // One elementary transposition P(batch, A, B, s): batch x [A x B x s] -> batch x [B x A x s]
 // (SURVEY.md R5).  The batch index T is split as T = to * inner + ti: item T starts at

@@ -44,6 +44,8 @@ struct TileParams {
     uint32_t buf_bytes;   // bytes of one smem tile buffer
     uint32_t nbuf;        // tma path: ring depth
     FastDiv divM, divN, divMV, divNV;  // m, n, m/V, n/V
+    FastDiv32 divM32, divN32;
+    int vec16;            // generic path: tiles 16-byte aligned, 16-byte loads
 };
 
 __device__ __forceinline__ char *tile_ptr(const TileParams &p, uint64_t t) {
@@ -206,22 +208,43 @@ __global__ void __launch_bounds__(512) tile_onchip_ldg(const TileParams p) {
 }
 
 // ------------------------------------------------------------------- generic kernel
+// Any element size and any m x n that fits (Fig. 1 for a CUDA block).  The tile is
+// contiguous, so when it is 16-byte aligned it is loaded with 16-byte vectors; elements
+// land in an odd-pitch shared array (conflict-free transposed reads) and are written
+// back with coalesced element stores (an output row of m elements is rarely 16-byte
+// aligned).  All index maps use 32-bit multiply-high division.
 template <typename T>
 __global__ void __launch_bounds__(512) tile_onchip_generic(const TileParams p) {
+    constexpr int PV = 16 / sizeof(T) > 0 ? 16 / sizeof(T) : 1;   // elements per 16 B
     extern __shared__ __align__(128) unsigned char smem_raw[];
     T *s = reinterpret_cast<T *>(smem_raw);
     const uint32_t mn = p.m * p.n;
     for (uint64_t t = blockIdx.x; t < p.count; t += gridDim.x) {
         T *g = reinterpret_cast<T *>(tile_ptr(p, t));
-        for (uint32_t e = threadIdx.x; e < mn; e += blockDim.x) {
-            uint64_t i, j;
-            fdivmod(e, p.divN, i, j);
-            s[i * p.pitch + j] = g[e];
+        if (p.vec16) {
+            const uint32_t nvec = mn / PV;
+            for (uint32_t e = threadIdx.x; e < nvec; e += blockDim.x) {
+                union { uint4 v; T x[PV]; } u;
+                u.v = ld_cg<16>(reinterpret_cast<const char *>(g) + (size_t)e * 16);
+                uint32_t i, j;
+                fdivmod32(e * PV, p.divN32, i, j);
+#pragma unroll
+                for (int k = 0; k < PV; ++k) {
+                    s[i * p.pitch + j] = u.x[k];
+                    if (++j == p.n) { j = 0; ++i; }
+                }
+            }
+        } else {
+            for (uint32_t e = threadIdx.x; e < mn; e += blockDim.x) {
+                uint32_t i, j;
+                fdivmod32(e, p.divN32, i, j);
+                s[i * p.pitch + j] = g[e];
+            }
         }
         __syncthreads();
         for (uint32_t o = threadIdx.x; o < mn; o += blockDim.x) {
-            uint64_t r, c;
-            fdivmod(o, p.divM, r, c);    // output row r < n, column c < m
+            uint32_t r, c;
+            fdivmod32(o, p.divM32, r, c);   // output row r < n, column c < m
             g[o] = s[c * p.pitch + r];
         }
         __syncthreads();
@@ -234,8 +257,9 @@ namespace {
 enum { MODE_LDG = 0, MODE_TMA = 1 };
 
 int tile_mode() { return (int)env_int("IPT_TILE_MODE", MODE_LDG); }
-int tile_threads() {
-    long t = env_int("IPT_TILE_THREADS", 512);
+int tile_threads(uint64_t tile_bytes) {
+    // small tiles: 256 threads (fewer idle threads in the write-out), else 512
+    long t = env_int("IPT_TILE_THREADS", tile_bytes < 48 * 1024 ? 256 : 512);
     return (t == 256 || t == 512) ? (int)t : 512;
 }
 uint32_t tma_nbuf() {
@@ -297,7 +321,7 @@ int occupancy(K kern, int threads, size_t smem, int device) {
 template <typename K>
 cudaError_t go(K kern, const TileParams &p, size_t smem, cudaStream_t st, int device) {
     DevProps dp = dev_props(device);
-    const int threads = tile_threads();
+    const int threads = tile_threads(p.tile_bytes);
     int per_sm = occupancy(kern, threads, smem, device);
     uint64_t grid = (uint64_t)dp.sms * per_sm;
     if (p.count < grid) grid = p.count;
@@ -357,6 +381,10 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
         }
     }
     p.pitch = generic_pitch(d.B);
+    p.divM32 = make_fastdiv32((uint32_t)d.A);
+    p.divN32 = make_fastdiv32((uint32_t)d.B);
+    p.vec16 = (((uintptr_t)d.base & 15) == 0) && (p.tile_bytes % 16 == 0) &&
+              (d.outer <= 1 || (d.ostride & 15) == 0) && d.eb <= 16;
     const size_t smem = generic_smem(d.A, d.B, d.eb);
     if ((long)smem > budget) return cudaErrorInvalidValue;
     switch (d.eb) {

@@ -80,6 +80,16 @@ def test_fastdiv_exact():
             assert L.ipt__fastdiv(n, d) == n // d, (n, d)
 
 
+def test_fastdiv32_exact():
+    L = ipt.lib()
+    rnd = random.Random(4)
+    ds = [1, 2, 3, 7, 131, 4999, 14803, 65536, 2**31 - 1, 2**31, 2**32 - 1]
+    for d in ds:
+        for n in [0, 1, d - 1, d, d + 1, 2**32 - 1, 2**31] + [rnd.randrange(2**32) for _ in range(300)]:
+            n &= 0xFFFFFFFF
+            assert L.ipt__fastdiv32(n, d) == n // d, (n, d)
+
+
 # ----------------------------------------------------------------------------- planner
 def _np_stages(a, M, N, m, n):
     Mp, Np = M // m, N // n
@@ -133,9 +143,10 @@ def test_plan_overhead_below_paper_bound():
 
 def test_plan_prefers_vector_tiles_on_large_f32():
     """Sec. 7.4 pruning: big super-elements for stages 1/3, tile on chip for stage 2."""
-    for (M, N) in [(7200, 1800), (16384, 16384), (20000, 20000)]:
+    for (M, N) in [(18000, 7200), (16384, 16384), (20000, 20000), (12800, 15000)]:
         p = ipt.plan(M, N, 4)
         assert p.n * 4 >= 256 and p.m * 4 >= 256
+        assert p.n * 4 % 64 == 0 and p.m * 4 % 64 == 0     # line-friendly super-elements
         assert ipt.VARIANTS[p.variant[1]] == "tile_onchip"
         assert p.n_stages == 3
 

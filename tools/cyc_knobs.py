@@ -17,12 +17,14 @@ def bench(batch, A, B, s, reps=3):
     e1.record(); torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / (2 * reps)
     return round(2 * batch * A * B * s * 4 / (ms / 1e3) / 1e9)
-knobs = [dict(IPT_CYC_SCRAMBLE="0"), dict(), dict(IPT_CYC_FENCE="0"),
-         dict(IPT_CYC_G="8", IPT_CYC_R="4"), dict(IPT_CYC_G="8", IPT_CYC_R="4", IPT_CYC_FENCE="0")]
+import ast
+knobs = ast.literal_eval(os.environ.get("KNOBS", "[{}]"))
 for kn in knobs:
     for k in list(os.environ):
         if k.startswith("IPT_CYC"): del os.environ[k]
     os.environ.update(kn)
     res = {"S512_st1": bench(1, 12800, 15000 // 128, 128), "S512_st3": bench(75, 100, 200, 128),
-           "S320_st3": bench(75, 160, 200, 80), "S800_st3": bench(75, 64, 200, 200), "S240_st1": bench(1, 12800, 250, 60)}
+           "S320_st3": bench(75, 160, 200, 80), "S800_st3": bench(75, 64, 200, 200), "S240_st1": bench(1, 12800, 250, 60),
+           "pow2_S512_st1": bench(1, 16384, 64, 128), "pow2_S512_st3": bench(64, 128, 128, 128),
+           "S576_st1": bench(1, 7200, 125, 144), "S640_st3": bench(125, 45, 144, 160)}
     print(json.dumps(kn), json.dumps(res), flush=True)

@@ -27,6 +27,7 @@
 #include "ipt_internal.h"
 #include "mem_ptx.cuh"
 
+#include <cstdio>
 #include <map>
 #include <mutex>
 
@@ -44,7 +45,8 @@ struct TileParams {
     uint32_t buf_bytes;   // bytes of one smem tile buffer
     uint32_t nbuf;        // tma path: ring depth
     FastDiv divM, divN, divMV, divNV;  // m, n, m/V, n/V
-    FastDiv32 divM32, divN32;
+    FastDiv32 divM32, divN32, divMV32, divMVK32, divNV32;   // m, n, m/V, (m/V)/K, n/V
+    uint32_t K;           // cluster path: CTAs per tile
     int vec16;            // generic path: tiles 16-byte aligned, 16-byte loads
 };
 
@@ -101,22 +103,26 @@ __device__ __forceinline__ void sts128(uint32_t saddr, const uint4 &v) {
 }
 
 // Write the transposed tile from padded shared memory (sbase, pitch q) to global g.
+// Only block rows [bi0, bi0 + mvp) of the tile (in V-row units) are in this CTA's shared
+// memory (row bil*V of the buffer holds tile row (bi0 + bil)*V): the whole tile for the
+// single-CTA kernels, one slice for the cluster kernel.
 template <int EB>
-__device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, char *g) {
+__device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, char *g,
+                                          uint32_t bi0, uint32_t mvp, const FastDiv32 &divmvp) {
     constexpr int V = 16 / EB;
     constexpr int ROT = (V >= 8) ? 1 : 8 / V;   // lanes sharing one rotation
     using E = typename Elem<EB>::T;
-    const uint32_t nblk = (p.m / V) * (p.n / V);
+    const uint32_t nblk = mvp * (p.n / V);
     for (uint32_t blk = threadIdx.x; blk < nblk; blk += blockDim.x) {
-        uint64_t bj64, bi64;
-        fdivmod(blk, p.divMV, bj64, bi64);
-        const uint32_t bi = (uint32_t)bi64, bj = (uint32_t)bj64;
-        const int off = (int)((bi / ROT) % V);
+        uint32_t bj, bil;
+        fdivmod32(blk, divmvp, bj, bil);
+        const uint32_t bi = bi0 + bil;
+        const int off = (int)((bil / ROT) % V);
         E x[V][V];
 #pragma unroll
         for (int kk = 0; kk < V; ++kk) {
             const uint32_t rho = (uint32_t)((kk + off) % V);
-            const uint4 v = lds128(sbase + ((bi * V + rho) * p.q + bj) * 16);
+            const uint4 v = lds128(sbase + ((bil * V + rho) * p.q + bj) * 16);
             unpack<EB>(v, x[kk]);
         }
         // x[kk][c] = tile[bi*V + (kk+off)%V][bj*V + c]; output row bj*V+c gets column c.
@@ -129,6 +135,11 @@ __device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, c
             stg128_na(g + ((size_t)(bj * V + c) * p.m + (size_t)bi * V) * EB, pack<EB>(col));
         }
     }
+}
+
+template <int EB>
+__device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, char *g) {
+    write_out<EB>(p, sbase, g, 0, p.m / (16 / EB), p.divMV32);
 }
 
 // ------------------------------------------------------------------- TMA ring kernel
@@ -178,7 +189,7 @@ __global__ void __launch_bounds__(512) tile_onchip_tma(const TileParams p) {
 
 // ------------------------------------------------------------ register-staged kernel
 template <int EB, int U>
-__global__ void __launch_bounds__(512) tile_onchip_ldg(const TileParams p) {
+__global__ void __launch_bounds__(512, 2) tile_onchip_ldg(const TileParams p) {
     extern __shared__ __align__(128) unsigned char smem[];
     const uint32_t sbase = smem_u32(smem);
     const uint32_t nvec = (uint32_t)(p.tile_bytes / 16);
@@ -195,15 +206,71 @@ __global__ void __launch_bounds__(512) tile_onchip_ldg(const TileParams p) {
             for (int u = 0; u < U; ++u) {
                 const uint32_t e = e0 + u * blockDim.x;
                 if (e < nvec) {
-                    uint64_t i, j;
-                    fdivmod(e, p.divNV, i, j);
-                    sts128(sbase + ((uint32_t)i * p.q + (uint32_t)j) * 16, v[u]);
+                    uint32_t i, j;
+                    fdivmod32(e, p.divNV32, i, j);
+                    sts128(sbase + (i * p.q + j) * 16, v[u]);
                 }
             }
         }
         __syncthreads();
         write_out<EB>(p, sbase, g);
         __syncthreads();
+    }
+}
+
+// -------------------------------------------------------------- cluster-split kernel
+// Tiles larger than one CTA's shared memory: a thread-block cluster of K CTAs (K SMs)
+// owns one tile; CTA k holds tile rows [k*m/K, (k+1)*m/K) and writes exactly the output
+// columns those rows become (every output row is [slice 0 | slice 1 | ... ]), so no
+// distributed-shared-memory traffic is needed.  The only cross-CTA hazard is in-place:
+// no CTA may store into the tile before every CTA of the cluster has finished loading
+// it -- one cluster barrier (release/acquire) per tile.  This lifts the paper's on-chip
+// tile limit to K x 227 KB, which lets stages 1 and 3 use larger
+// super-elements.
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+template <int EB, int U>
+__global__ void __launch_bounds__(512, 2) tile_onchip_cluster(const TileParams p) {
+    constexpr int V = 16 / EB;
+    extern __shared__ __align__(128) unsigned char smem[];
+    const uint32_t sbase = smem_u32(smem);
+    const uint32_t K = p.K;
+    const uint32_t rank = cluster_rank();
+    const uint32_t cid = blockIdx.x / K, ncl = gridDim.x / K;
+    const uint32_t rows = p.m / K;                 // tile rows held by this CTA
+    const uint32_t nvrow = p.n / V;                // 16-byte vectors per row
+    const uint32_t nvec = rows * nvrow;
+    const size_t slice_off = (size_t)rank * rows * p.n * EB;
+    for (uint64_t t = cid; t < p.count; t += ncl) {
+        char *g = tile_ptr(p, t);
+        const char *src = g + slice_off;
+        for (uint32_t e0 = threadIdx.x; e0 < nvec; e0 += U * blockDim.x) {
+            uint4 v[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const uint32_t e = e0 + u * blockDim.x;
+                if (e < nvec) v[u] = ld_cg<16>(src + (size_t)e * 16);
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const uint32_t e = e0 + u * blockDim.x;
+                if (e < nvec) {
+                    uint32_t i, j;
+                    fdivmod32(e, p.divNV32, i, j);
+                    sts128(sbase + (i * p.q + j) * 16, v[u]);
+                }
+            }
+        }
+        cluster_sync_all();     // every slice of tile t is on chip before anyone stores
+        write_out<EB>(p, sbase, g, rank * (rows / V), rows / V, p.divMVK32);
+        __syncthreads();        // shared slice consumed before the next tile's loads
     }
 }
 
@@ -331,12 +398,69 @@ cudaError_t go(K kern, const TileParams &p, size_t smem, cudaStream_t st, int de
     return cudaGetLastError();
 }
 
+template <typename K_>
+cudaError_t go_cluster(K_ kern, const TileParams &p, size_t smem, int K, cudaStream_t st,
+                       int device) {
+    DevProps dp = dev_props(device);
+    const int threads = tile_threads(smem);
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dp.smem_optin);
+    cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    cudaLaunchConfig_t cfg = {};
+    cfg.blockDim = dim3(threads, 1, 1);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = K;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    int per_sm = occupancy(kern, threads, smem, device);
+    uint64_t clusters = (uint64_t)dp.sms * per_sm / K;
+    cfg.gridDim = dim3((unsigned)(clusters * K), 1, 1);
+    int maxc = 0;   // co-resident clusters (cluster placement may strand SMs)
+    if (cudaOccupancyMaxActiveClusters(&maxc, kern, &cfg) == cudaSuccess && maxc > 0) {
+        if ((uint64_t)maxc < clusters && (uint64_t)maxc * 2 >= clusters) clusters = (uint64_t)maxc;
+    } else {
+        cudaGetLastError();
+    }
+    if (p.count < clusters) clusters = p.count;
+    if (clusters < 1) clusters = 1;
+    cfg.gridDim = dim3((unsigned)(clusters * K), 1, 1);
+    if (env_int("IPT_DEBUG", 0))
+        fprintf(stderr, "[ipt] tile_cluster K=%d smem=%zu threads=%d per_sm=%d maxc=%d clusters=%llu tiles=%llu\n",
+                K, smem, threads, per_sm, maxc, (unsigned long long)clusters, (unsigned long long)p.count);
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, p);
+    note_launch();
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
+
 }  // namespace
+
+// Cluster size for a tile that does not fit one CTA (0 = none): the smallest K in
+// {2, 4, 8} whose row slice fits 113 KB (two CTAs per SM), else the smallest that fits.
+int tile_cluster_k(int64_t A, int64_t B, int eb, int device) {
+    if (!vec_ok(A, B, eb) || !env_int("IPT_TILE_CLUSTER", 1)) return 0;
+    DevProps dp = dev_props(device);
+    const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
+    const int V = 16 / eb;
+    const size_t rowb = (size_t)fast_q(B, eb) * 16;
+    int fit = 0;
+    for (int K : {2, 4, 8}) {
+        if (A % (K * V)) continue;
+        const size_t slice = (size_t)(A / K) * rowb;
+        if (slice <= 113 * 1024) return K;
+        if (!fit && (long)slice <= budget) fit = K;
+    }
+    return fit;
+}
 
 int tile_onchip_path(int64_t A, int64_t B, int eb, int device) {
     DevProps dp = dev_props(device);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
     if (vec_ok(A, B, eb) && (long)fast_smem(A, B, eb) <= budget) return 2;
+    if (tile_cluster_k(A, B, eb, device)) return 3;
     if ((long)generic_smem(A, B, eb) <= budget && A * B < (1ll << 31)) return 1;
     return 0;
 }
@@ -364,6 +488,8 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
         p.buf_bytes = (uint32_t)((size_t)d.A * p.q * 16);
         p.divMV = make_fastdiv((uint64_t)(d.A / V));
         p.divNV = make_fastdiv((uint64_t)(d.B / V));
+        p.divNV32 = make_fastdiv32((uint32_t)(d.B / V));
+        p.divMV32 = make_fastdiv32((uint32_t)(d.A / V));
         p.nbuf = tma_nbuf();
         const size_t smem = fast_smem(d.A, d.B, d.eb);
         if (tile_mode() == MODE_TMA) {
@@ -377,6 +503,22 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
                 case 4: return go(tile_onchip_ldg<4, 8>, p, smem, st, device);
                 case 8: return go(tile_onchip_ldg<8, 8>, p, smem, st, device);
                 case 16: return go(tile_onchip_ldg<16, 8>, p, smem, st, device);
+            }
+        }
+    }
+    if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) > budget) {
+        const int K = tile_cluster_k(d.A, d.B, d.eb, device);
+        if (K) {
+            const int V = 16 / d.eb;
+            p.q = fast_q(d.B, d.eb);
+            p.K = (uint32_t)K;
+            p.divMVK32 = make_fastdiv32((uint32_t)(d.A / V / K));
+            p.divNV32 = make_fastdiv32((uint32_t)(d.B / V));
+            const size_t smem = (size_t)(d.A / K) * p.q * 16;
+            switch (d.eb) {
+                case 4: return go_cluster(tile_onchip_cluster<4, 8>, p, smem, K, st, device);
+                case 8: return go_cluster(tile_onchip_cluster<8, 8>, p, smem, K, st, device);
+                case 16: return go_cluster(tile_onchip_cluster<16, 8>, p, smem, K, st, device);
             }
         }
     }

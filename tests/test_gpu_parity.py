@@ -386,3 +386,15 @@ def test_transpose_host_queues(queues):
         assert tuple(out.shape) == (N, M)
         ref = oracle.transpose_inplace(a.copy(), M, N)
         assert np.array_equal(h.numpy().view(np.uint32), ref), (M, N, queues)
+
+
+# ------------------------------------------------- cluster-split tiles (> 227 KB)
+@pytest.mark.parametrize("eb,batch,A,B", [(4, 3, 512, 512), (4, 2, 7200 // 4, 60), (4, 5, 640, 600),
+                                          (8, 3, 400, 400), (16, 2, 256, 256), (4, 7, 960, 400)])
+def test_ipt_010_cluster_tiles(eb, batch, A, B):
+    """Tiles larger than one CTA's shared memory are split over a thread-block cluster
+    (one barrier.cluster per tile); bit-exact vs the oracle."""
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)

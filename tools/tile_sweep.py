@@ -18,8 +18,8 @@ def bench(m, n, reps=5):
     e1.record(); torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / (2 * reps)
     return 2 * cnt * m * n * 4 / (ms / 1e3) / 1e9
-shapes = [(128, 200), (160, 160), (100, 100), (64, 200), (128, 128), (160, 144), (128, 256), (256, 200), (200, 256), (240, 240), (80, 240), (120, 480)]
-for mode, thr, st in [("0", "512", "2"), ("0", "256", "2")]:
+shapes = [(128, 200), (160, 160), (64, 200), (256, 256), (320, 320), (400, 400), (512, 512), (640, 600), (800, 400), (960, 400), (720, 288), (200, 512), (7200 // 4, 60), (160, 800), (1600, 256)]
+for mode, thr, st in [("0", "512", "2")]:
     os.environ["IPT_TILE_MODE"] = mode; os.environ["IPT_TILE_THREADS"] = thr; os.environ["IPT_TILE_STAGES"] = st
     res = {}
     for (m, n) in shapes:

@@ -282,10 +282,179 @@ cycle_global_kernel(const CycParams p) {
     }
 }
 
+// ------------------------------------------------------------ unaligned super-elements
+// Super-elements whose size is a multiple of 4 but not of 16 bytes (e.g. m = 131 floats):
+// their start addresses have different 16-byte phases, so the carried data cannot keep a
+// fixed lane/vector mapping.  A warp walker (G = 32) loads the 16-byte vectors COVERING
+// the target, keeps the carried super-element word-aligned in a per-warp shared buffer,
+// and writes it back realigned: whole 16-byte vectors inside, per-word stores at the two
+// partial ends.  Same claim protocol and start schedule as cycle_global_kernel.
+template <int R, typename I>
+__global__ void __launch_bounds__(256, 6) cycle_ua_kernel(const CycParams p) {
+    constexpr unsigned FULL = 0xffffffffu;
+    __shared__ uint32_t carry_all[8][R * 128];
+    const int lane = threadIdx.x & 31;
+    uint32_t *carry = carry_all[threadIdx.x >> 5];
+    const I A = (I)p.A, nchunk = (I)p.nchunk, nwords = (I)p.nwords;
+
+    int mode = M_FETCH;
+    I word = 0;
+    uint32_t cw = 0;
+    int nb = 0;
+    char *item = nullptr;
+    I ubase = 0, k = 0, k0 = 0;
+    int nw = 0;                          // 4-byte words in this chunk
+    uint4 in[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) in[r] = make_uint4(0, 0, 0, 0);
+
+    for (;;) {
+        // ------------------------------------------------ work acquisition (warp-uniform)
+        for (; mode == M_FETCH || mode == M_SCAN;) {
+            if (mode == M_FETCH) {
+                unsigned long long wb = 0;
+                if (lane == 0) wb = atomicAdd(p.counter, 1ull);
+                wb = __shfl_sync(FULL, wb, 0);
+                if (wb >= p.nwords) { mode = M_DONE; break; }
+                uint64_t mine = wb;
+                if (p.wstride != 1) {
+                    uint64_t q, r;
+                    fdivmod(wb * p.wstride, p.divNwords.d64, q, r);
+                    mine = r;
+                }
+                word = (I)mine;
+                cw = ld_relaxed_u32(p.flags + word);
+                cw = __shfl_sync(FULL, cw, 0);
+                nb = 0;
+                mode = M_SCAN;
+            }
+            uint32_t valid = 0xffffffffu;
+            if (word == nwords - 1 && (p.units & 31)) valid = (1u << (p.units & 31)) - 1u;
+            const uint32_t cand = ~cw & valid & (nb >= 32 ? 0u : (0xffffffffu << nb));
+            if (!cand) { mode = M_FETCH; continue; }
+            const int b = __ffs(cand) - 1;
+            nb = b + 1;
+            const I u = word * 32 + (I)b;
+            I tk = u, ch = 0;
+            if (p.nchunk > 1) fdivmod_t(u, p.divNchunk.d32, p.divNchunk.d64, tk, ch);
+            I T, kk, q, r;
+            fdivmod_t(tk, p.divAB.d32, p.divAB.d64, T, kk);
+            fdivmod_t(kk, p.divB.d32, p.divB.d64, q, r);
+            if (r * A + q == kk) continue;              // fixed point of Eq. (1)
+            I to, ti;
+            fdivmod_t(T, p.divInner.d32, p.divInner.d64, to, ti);
+            item = p.base + (uint64_t)to * p.ostride + (uint64_t)ti * p.istride +
+                   (uint64_t)ch * p.cvec * 4;
+            ubase = T * (I)p.AB * nchunk + ch;
+            nw = (int)((ch == nchunk - 1) ? (p.nvec - (uint64_t)ch * p.cvec) : p.cvec);
+            k = k0 = kk;
+            mode = M_START;
+            break;
+        }
+        if (mode == M_DONE) break;
+
+        // --------------------------------------------------------------- memory round
+        I tgt = k;
+        if (mode == M_CHAIN) {
+            I q, r;
+            fdivmod_t(k, p.divB.d32, p.divB.d64, q, r);
+            tgt = r * A + q;
+        }
+        const bool back_home = (mode == M_CHAIN) && (tgt == k0);
+        const I ut = ubase + tgt * nchunk;
+        const uint32_t bit = 1u << ((uint32_t)ut & 31);
+        uint32_t *fwp = p.flags + (ut >> 5);
+        const uintptr_t a = (uintptr_t)(item + (uint64_t)tgt * p.S);
+        const int o = (int)((a & 15) >> 2);             // word phase of the target
+        const char *vb = (const char *)(a - (uintptr_t)(o * 4));
+        const int nvv = (o + nw + 3) >> 2;              // covering 16-byte vectors
+        if ((mode == M_START || mode == M_CHAIN) && !back_home) {
+#pragma unroll
+            for (int r = 0; r < R; ++r) {
+                const int j = lane + 32 * r;
+                if (j < nvv) in[r] = ld_cg<16>(vb + (size_t)j * 16);
+            }
+        }
+        uint32_t old = 0;
+        if (mode == M_CHAIN && lane == 0)
+            old = p.fence ? atom_or_acq_u32(fwp, bit) : atom_or_u32(fwp, bit);
+        uint32_t fw = 0;
+        if (mode == M_START) {
+            if (p.fence) fence_acq_rel_gpu();
+            fw = ld_relaxed_u32(fwp);
+        } else if (mode == M_REFRESH) {
+            fw = ld_relaxed_u32(p.flags + word);
+        }
+        old = __shfl_sync(FULL, old, 0);
+        __syncwarp();
+        const bool start_lost = __any_sync(FULL, (fw & bit) != 0);
+
+        auto carry_from_in = [&]() {            // carry[t] = word t of the loaded target
+            __syncwarp();
+#pragma unroll
+            for (int r = 0; r < R; ++r) {
+                const int j = lane + 32 * r;
+                if (j < nvv) {
+                    const uint32_t w4[4] = {in[r].x, in[r].y, in[r].z, in[r].w};
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const int t = 4 * j + i - o;
+                        if (t >= 0 && t < nw) carry[t] = w4[i];
+                    }
+                }
+            }
+            __syncwarp();
+        };
+
+        if (mode == M_START) {
+            cw |= fw;
+            if (start_lost) {
+                mode = M_SCAN;
+            } else {
+                carry_from_in();
+                mode = M_CHAIN;
+            }
+        } else if (mode == M_CHAIN) {
+            if (!(old & bit)) {
+                // store the carried words into the target, realigned to its phase o
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    const int j = lane + 32 * r;
+                    if (j < nvv) {
+                        char *dst = (char *)vb + (size_t)j * 16;
+                        const int t0 = 4 * j - o;
+                        if (t0 >= 0 && t0 + 3 < nw) {
+                            st_cg<16>(dst, make_uint4(carry[t0], carry[t0 + 1], carry[t0 + 2], carry[t0 + 3]));
+                        } else {
+#pragma unroll
+                            for (int i = 0; i < 4; ++i) {
+                                const int t = t0 + i;
+                                if (t >= 0 && t < nw) st_cg<4>(dst + 4 * i, carry[t]);
+                            }
+                        }
+                    }
+                }
+                if (back_home) {
+                    __syncwarp();
+                    mode = M_SCAN;
+                } else {
+                    carry_from_in();            // the displaced content is carried on
+                    k = tgt;
+                }
+            } else {
+                mode = p.refresh ? M_REFRESH : M_SCAN;
+            }
+        } else if (mode == M_REFRESH) {
+            cw |= fw;
+            mode = M_SCAN;
+        }
+    }
+}
+
 // ------------------------------------------------------------------------- host side
 namespace {
 
-struct Choice { int W, G, R; uint64_t cvec, nchunk; };
+struct Choice { int W, G, R; uint64_t cvec, nchunk; bool ua; };
 
 int pick_vec_bytes(const StageDesc &d) {
     const uint64_t S = (uint64_t)d.s * d.eb;
@@ -301,6 +470,18 @@ Choice choose(const StageDesc &d) {
     Choice c;
     const uint64_t S = (uint64_t)d.s * d.eb;
     c.W = pick_vec_bytes(d);
+    c.ua = false;
+    if ((c.W == 4 || c.W == 8) && S >= 64 && env_int("IPT_CYC_UA", 1)) {
+        // 4-byte granular super-elements with mixed 16-byte phases: realigning walker
+        c.ua = true;
+        c.W = 4;
+        const uint64_t nw = S / 4;
+        c.nchunk = (nw + 508) / 509;
+        c.cvec = (nw + c.nchunk - 1) / c.nchunk;              // words per chunk
+        c.G = 32;
+        c.R = c.cvec <= 125 ? 1 : (c.cvec <= 253 ? 2 : 4);
+        return c;
+    }
     const uint64_t nvec = S / c.W;
     const long max_chunk = env_int("IPT_CYC_MAXVEC", 128);   // vectors per walker chunk
     uint64_t cap = (uint64_t)(max_chunk < 1 ? 1 : max_chunk);
@@ -361,6 +542,33 @@ cudaError_t launch_t(const CycParams &p, cudaStream_t st, int device) {
     return cudaGetLastError();
 }
 
+template <int R, typename I>
+cudaError_t launch_ua(const CycParams &p, cudaStream_t st, int device) {
+    auto kern = cycle_ua_kernel<R, I>;
+    static std::mutex mu;
+    static std::map<int, int> occ_cache;
+    int per_sm = 0;
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = occ_cache.find(device);
+        if (it == occ_cache.end()) {
+            cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 256, 0);
+            if (e != cudaSuccess) return e;
+            occ_cache[device] = per_sm;
+        } else {
+            per_sm = it->second;
+        }
+    }
+    DevProps dp = dev_props(device);
+    uint64_t grid = (uint64_t)dp.sms * (uint64_t)(per_sm > 0 ? per_sm : 1);
+    const uint64_t need = (p.nwords + 7) / 8;
+    if (need < grid) grid = need;
+    if (grid < 1) grid = 1;
+    kern<<<(unsigned)grid, 256, 0, st>>>(p);
+    note_launch();
+    return cudaGetLastError();
+}
+
 typedef cudaError_t (*LaunchFn)(const CycParams &, cudaStream_t, int);
 
 template <int W, int G, int R>
@@ -372,6 +580,11 @@ LaunchFn pick_idx(bool idx32) {
     if (c.W == W_ && c.G == G_ && c.R == R_) return pick_idx<W_, G_, R_>(idx32);
 
 LaunchFn lookup(const Choice &c, bool idx32) {
+    if (c.ua) {
+        if (c.R == 1) return idx32 ? &launch_ua<1, uint32_t> : &launch_ua<1, uint64_t>;
+        if (c.R == 2) return idx32 ? &launch_ua<2, uint32_t> : &launch_ua<2, uint64_t>;
+        return idx32 ? &launch_ua<4, uint32_t> : &launch_ua<4, uint64_t>;
+    }
     // W = 16: every group width
     IPT_CASE(16, 1, 1) IPT_CASE(16, 2, 1) IPT_CASE(16, 4, 1) IPT_CASE(16, 8, 1)
     IPT_CASE(16, 16, 1) IPT_CASE(16, 32, 1) IPT_CASE(16, 32, 2) IPT_CASE(16, 32, 4)

@@ -398,3 +398,16 @@ def test_ipt_010_cluster_tiles(eb, batch, A, B):
     t = to_dev(a, eb)
     ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
     assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)
+
+
+# ---------------------------------------- unaligned super-elements (S % 16 != 0)
+@pytest.mark.parametrize("batch,A,B,s,eb", [(1, 61, 47, 131, 4), (3, 20, 30, 17, 4), (2, 9, 11, 4999, 4),
+                                            (4, 33, 31, 65, 4), (1, 50, 70, 63, 8), (2, 40, 44, 1001, 8),
+                                            (1, 256, 131, 131, 4)])
+def test_ipt_100_unaligned_realigning_walker(batch, A, B, s, eb):
+    """4-byte-granular super-elements whose start phases differ mod 16 B use the
+    realigning warp walker (covering 16-B loads, shared-memory carry, partial stores)."""
+    a = gen(batch * A * B * s, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_100_(t, batch, A, B, s)
+    assert np.array_equal(to_np(t, eb), oracle.permute_inplace(a.copy(), batch, A, B, s))

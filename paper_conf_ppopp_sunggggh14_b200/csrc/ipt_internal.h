@@ -87,7 +87,8 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
 // and an A x B tile must fit in shared memory (tile_onchip_fits()).
 bool tile_onchip_fits(int64_t A, int64_t B, int eb, int device);
 // 0: does not fit, 1: generic element path, 2: 16-byte path in one CTA,
-// 3: 16-byte path split over a thread-block cluster (tile_cluster_k CTAs)
+// 3: 16-byte path split over a thread-block cluster (tile_cluster_k CTAs),
+// 4: element path split over a thread-block cluster
 int tile_onchip_path(int64_t A, int64_t B, int eb, int device);
 int tile_cluster_k(int64_t A, int64_t B, int eb, int device);
 cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device);

@@ -47,6 +47,7 @@ struct TileParams {
     FastDiv divM, divN, divMV, divNV;  // m, n, m/V, n/V
     FastDiv32 divM32, divN32, divMV32, divMVK32, divNV32;   // m, n, m/V, (m/V)/K, n/V
     uint32_t K;           // cluster path: CTAs per tile
+    int colsplit;         // generic cluster path: split columns (1) or rows (0)
     int vec16;            // generic path: tiles 16-byte aligned, 16-byte loads
 };
 
@@ -274,6 +275,61 @@ __global__ void __launch_bounds__(512, 2) tile_onchip_cluster(const TileParams p
     }
 }
 
+// Element loads of `cnt` contiguous elements (row length via divN) into an odd-pitch
+// shared array, U loads in flight per thread.
+template <typename T, int U = 8>
+__device__ __forceinline__ void load_slice_scalar(T *s, const T *src, uint32_t cnt, uint32_t pitch,
+                                                  const FastDiv32 &divN) {
+    for (uint32_t e0 = threadIdx.x; e0 < cnt; e0 += U * blockDim.x) {
+        T v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const uint32_t e = e0 + u * blockDim.x;
+            if (e < cnt) v[u] = src[e];
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const uint32_t e = e0 + u * blockDim.x;
+            if (e < cnt) {
+                uint32_t i, j;
+                fdivmod32(e, divN, i, j);
+                s[i * pitch + j] = v[u];
+            }
+        }
+    }
+}
+
+// Same with 16-byte vector loads (src 16-byte aligned, cnt * sizeof(T) % 16 == 0).
+template <typename T, int U = 4>
+__device__ __forceinline__ void load_slice_vec(T *s, const T *src, uint32_t cnt, uint32_t pitch,
+                                               uint32_t n, const FastDiv32 &divN) {
+    constexpr int PV = 16 / sizeof(T) > 0 ? 16 / sizeof(T) : 1;
+    const uint32_t nvec = cnt / PV;
+    for (uint32_t e0 = threadIdx.x; e0 < nvec; e0 += U * blockDim.x) {
+        uint4 v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const uint32_t e = e0 + u * blockDim.x;
+            if (e < nvec) v[u] = ld_cg<16>(reinterpret_cast<const char *>(src) + (size_t)e * 16);
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const uint32_t e = e0 + u * blockDim.x;
+            if (e < nvec) {
+                union { uint4 w; T x[PV]; } uu;
+                uu.w = v[u];
+                uint32_t i, j;
+                fdivmod32(e * PV, divN, i, j);
+#pragma unroll
+                for (int k = 0; k < PV; ++k) {
+                    s[i * pitch + j] = uu.x[k];
+                    if (++j == n) { j = 0; ++i; }
+                }
+            }
+        }
+    }
+}
+
 // ------------------------------------------------------------------- generic kernel
 // Any element size and any m x n that fits (Fig. 1 for a CUDA block).  The tile is
 // contiguous, so when it is 16-byte aligned it is loaded with 16-byte vectors; elements
@@ -302,11 +358,7 @@ __global__ void __launch_bounds__(512) tile_onchip_generic(const TileParams p) {
                 }
             }
         } else {
-            for (uint32_t e = threadIdx.x; e < mn; e += blockDim.x) {
-                uint32_t i, j;
-                fdivmod32(e, p.divN32, i, j);
-                s[i * p.pitch + j] = g[e];
-            }
+            load_slice_scalar<T>(s, g, mn, p.pitch, p.divN32);
         }
         __syncthreads();
         for (uint32_t o = threadIdx.x; o < mn; o += blockDim.x) {
@@ -315,6 +367,99 @@ __global__ void __launch_bounds__(512) tile_onchip_generic(const TileParams p) {
             g[o] = s[c * p.pitch + r];
         }
         __syncthreads();
+    }
+}
+
+// ------------------------------------------------------ cluster-split generic kernel
+// Element path for tiles larger than one CTA (e.g. m = 9998 = 2 x 4999 rows): CTA k of a
+// K-CTA cluster holds rows [k*m/K, (k+1)*m/K) (uneven slices allowed) and writes the
+// matching column segment of every output row with coalesced element stores.  One
+// cluster barrier per tile separates all loads of the tile from all stores into it.
+__device__ __forceinline__ FastDiv32 make_fastdiv32_dev(uint32_t d) {
+    FastDiv32 f;
+    if (d == 0) d = 1;
+    f.d = d;
+    const uint32_t l = (d > 1) ? 32 - __clz(d - 1) : 0;
+    const uint64_t two_l = (uint64_t)1 << l;
+    f.m = (uint32_t)((((two_l - d) << 32) / d) + 1);
+    f.s1 = l ? 1 : 0;
+    f.s2 = l ? l - 1 : 0;
+    return f;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(512, 1) tile_generic_cluster(const TileParams p) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    T *s = reinterpret_cast<T *>(smem_raw);
+    const uint32_t K = p.K;
+    const uint32_t rank = cluster_rank();
+    const uint32_t cid = blockIdx.x / K, ncl = gridDim.x / K;
+    if (!p.colsplit) {
+        // row split: CTA k holds rows [r0, r1); writes that column segment of every output row
+        const uint32_t r0 = (uint32_t)((uint64_t)rank * p.m / K);
+        const uint32_t r1 = (uint32_t)((uint64_t)(rank + 1) * p.m / K);
+        const uint32_t rows = r1 - r0;
+        const uint32_t cnt = rows * p.n;
+        const FastDiv32 divRows = make_fastdiv32_dev(rows);
+        const bool vec = p.vec16 && (((uint64_t)r0 * p.n * sizeof(T)) % 16 == 0) &&
+                         (((uint64_t)cnt * sizeof(T)) % 16 == 0);
+        for (uint64_t t = cid; t < p.count; t += ncl) {
+            T *g = reinterpret_cast<T *>(tile_ptr(p, t));
+            const T *src = g + (size_t)r0 * p.n;
+            if (vec)
+                load_slice_vec<T>(s, src, cnt, p.pitch, p.n, p.divN32);
+            else
+                load_slice_scalar<T>(s, src, cnt, p.pitch, p.divN32);
+            cluster_sync_all();     // all slices loaded before any store into the tile
+            for (uint32_t o = threadIdx.x; o < cnt; o += blockDim.x) {
+                uint32_t r, cl;
+                fdivmod32(o, divRows, r, cl);   // output row r < n, column r0 + cl
+                g[(size_t)r * p.m + r0 + cl] = s[cl * p.pitch + r];
+            }
+            __syncthreads();
+        }
+    } else {
+        // column split (few, long rows): CTA k holds columns [c0, c1) of every row and
+        // writes output rows [c0, c1) -- one contiguous range
+        const uint32_t c0 = (uint32_t)((uint64_t)rank * p.n / K);
+        const uint32_t c1 = (uint32_t)((uint64_t)(rank + 1) * p.n / K);
+        const uint32_t cols = c1 - c0;
+        const uint32_t P = cols | 1u;
+        const uint32_t cnt = p.m * cols;
+        const FastDiv32 divCols = make_fastdiv32_dev(cols);
+        for (uint64_t t = cid; t < p.count; t += ncl) {
+            T *g = reinterpret_cast<T *>(tile_ptr(p, t));
+            constexpr int U = 8;
+            for (uint32_t e0 = threadIdx.x; e0 < cnt; e0 += U * blockDim.x) {
+                T v[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const uint32_t e = e0 + u * blockDim.x;
+                    if (e < cnt) {
+                        uint32_t i, jl;
+                        fdivmod32(e, divCols, i, jl);
+                        v[u] = g[(size_t)i * p.n + c0 + jl];
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const uint32_t e = e0 + u * blockDim.x;
+                    if (e < cnt) {
+                        uint32_t i, jl;
+                        fdivmod32(e, divCols, i, jl);
+                        s[i * P + jl] = v[u];
+                    }
+                }
+            }
+            cluster_sync_all();
+            T *dst = g + (size_t)c0 * p.m;
+            for (uint32_t o = threadIdx.x; o < cnt; o += blockDim.x) {
+                uint32_t rl, c;
+                fdivmod32(o, p.divM32, rl, c);   // output row c0 + rl, column c
+                dst[o] = s[c * P + rl];
+            }
+            __syncthreads();
+        }
     }
 }
 
@@ -456,11 +601,38 @@ int tile_cluster_k(int64_t A, int64_t B, int eb, int device) {
     return fit;
 }
 
+// Cluster size for the element path when the tile does not fit one CTA (0 = none).
+// Row split by default (16-byte slice loads; measured faster even for 32 x 9998 tiles);
+// IPT_TILE_COLSPLIT=1 selects the column split for tiles with more columns than rows.
+static bool generic_colsplit(int64_t A, int64_t B) {
+    return env_int("IPT_TILE_COLSPLIT", 0) && B > A;
+}
+
+int tile_generic_cluster_k(int64_t A, int64_t B, int eb, int device) {
+    if (!env_int("IPT_TILE_CLUSTER", 1) || A * B >= (1ll << 31)) return 0;
+    DevProps dp = dev_props(device);
+    const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
+    const bool cs = generic_colsplit(A, B);
+    for (int K : {2, 4, 8}) {
+        size_t bytes;
+        if (cs) {
+            if (B < K) break;
+            bytes = (size_t)A * (size_t)(((B + K - 1) / K) | 1) * eb;
+        } else {
+            if (A < K) break;
+            bytes = (size_t)((A + K - 1) / K) * generic_pitch(B) * eb;
+        }
+        if ((long)bytes <= budget) return K;
+    }
+    return 0;
+}
+
 int tile_onchip_path(int64_t A, int64_t B, int eb, int device) {
     DevProps dp = dev_props(device);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
     if (vec_ok(A, B, eb) && (long)fast_smem(A, B, eb) <= budget) return 2;
     if (tile_cluster_k(A, B, eb, device)) return 3;
+    if ((long)generic_smem(A, B, eb) > budget && tile_generic_cluster_k(A, B, eb, device)) return 4;
     if ((long)generic_smem(A, B, eb) <= budget && A * B < (1ll << 31)) return 1;
     return 0;
 }
@@ -528,7 +700,23 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
     p.vec16 = (((uintptr_t)d.base & 15) == 0) && (p.tile_bytes % 16 == 0) &&
               (d.outer <= 1 || (d.ostride & 15) == 0) && d.eb <= 16;
     const size_t smem = generic_smem(d.A, d.B, d.eb);
-    if ((long)smem > budget) return cudaErrorInvalidValue;
+    if ((long)smem > budget) {
+        const int K = tile_generic_cluster_k(d.A, d.B, d.eb, device);
+        if (!K) return cudaErrorInvalidValue;
+        p.K = (uint32_t)K;
+        p.colsplit = generic_colsplit(d.A, d.B) ? 1 : 0;
+        const size_t cs = p.colsplit
+            ? (size_t)d.A * (size_t)(((d.B + K - 1) / K) | 1) * d.eb
+            : (size_t)((d.A + K - 1) / K) * p.pitch * d.eb;
+        switch (d.eb) {
+            case 1: return go_cluster(tile_generic_cluster<uint8_t>, p, cs, K, st, device);
+            case 2: return go_cluster(tile_generic_cluster<uint16_t>, p, cs, K, st, device);
+            case 4: return go_cluster(tile_generic_cluster<uint32_t>, p, cs, K, st, device);
+            case 8: return go_cluster(tile_generic_cluster<unsigned long long>, p, cs, K, st, device);
+            case 16: return go_cluster(tile_generic_cluster<uint4>, p, cs, K, st, device);
+        }
+        return cudaErrorInvalidValue;
+    }
     switch (d.eb) {
         case 1: return go(tile_onchip_generic<uint8_t>, p, smem, st, device);
         case 2: return go(tile_onchip_generic<uint16_t>, p, smem, st, device);

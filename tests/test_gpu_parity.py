@@ -411,3 +411,23 @@ def test_ipt_100_unaligned_realigning_walker(batch, A, B, s, eb):
     t = to_dev(a, eb)
     ipt.ipt_100_(t, batch, A, B, s)
     assert np.array_equal(to_np(t, eb), oracle.permute_inplace(a.copy(), batch, A, B, s))
+
+
+@pytest.mark.parametrize("eb,batch,A,B", [(4, 2, 4999, 32), (4, 3, 1999, 31), (8, 2, 3001, 17),
+                                          (2, 2, 997, 301), (4, 1, 9998, 24)])
+def test_ipt_010_generic_cluster_tiles(eb, batch, A, B):
+    """Element-path tiles larger than one CTA: uneven row slices over a cluster."""
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)
+
+
+@pytest.mark.parametrize("eb,batch,A,B", [(4, 2, 32, 9998), (4, 3, 24, 4999), (8, 2, 17, 3001), (1, 2, 7, 40001)])
+def test_ipt_010_generic_cluster_column_split(monkeypatch, eb, batch, A, B):
+    """Few long rows: each cluster CTA owns a column range, writes whole output rows."""
+    monkeypatch.setenv("IPT_TILE_COLSPLIT", "1")
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)

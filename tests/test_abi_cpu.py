@@ -146,7 +146,7 @@ def test_plan_prefers_vector_tiles_on_large_f32():
     for (M, N) in [(18000, 7200), (16384, 16384), (20000, 20000), (12800, 15000)]:
         p = ipt.plan(M, N, 4)
         assert p.n * 4 >= 256 and p.m * 4 >= 256
-        assert p.n * 4 % 32 == 0 and p.m * 4 % 32 == 0     # sector-aligned super-elements
+        assert p.n * 4 % 16 == 0 and p.m * 4 % 16 == 0     # 16-byte vector super-elements
         assert ipt.VARIANTS[p.variant[1]] == "tile_onchip"
         assert p.n_stages == 3
 

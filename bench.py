@@ -190,6 +190,7 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_ppopp_sunggggh14_b200 as ipt
+    from paper_conf_ppopp_sunggggh14_b200.partition import shard
     from inputs import seeded
 
     assert args.warmup >= 3, "timing rules: at least 3 warm-up steps"
@@ -207,7 +208,7 @@ def main():
     if "batch" in wl:
         M, N = wl["shapes"][0]
         tot = wl["batch"]
-        lo, hi = tot * rank // world, tot * (rank + 1) // world
+        lo, hi = shard(tot, world, rank)          # contiguous block of matrices per rank
         t = torch.empty((hi - lo) * M * N, dtype=tdt, device=dev)
         seeded.fill_device_(t, M, N, eb, t0=lo, count=hi - lo)
         mats.append([t, M, N, hi - lo, lo])

@@ -180,6 +180,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--queues", type=int, default=4)
+    ap.add_argument("--algo", default="3stage", choices=["3stage", "4stage"],
+                    help="4stage = the paper's Gustavson/Karlsson baseline (comparison only)")
     args = ap.parse_args()
     world, rank, local = dist_setup()
 
@@ -232,6 +234,8 @@ def main():
             p = plans[(a, b)]
             if cnt > 1:
                 ipt.transpose_batched_(t, cnt, a, b, plan_=p)
+            elif args.algo == "4stage":      # the paper's 4-stage baseline
+                ipt.transpose_4stage_(t, a, b, p.m, p.n)
             else:
                 ipt.transpose_(t, a, b, plan_=p, workspace=ws,
                                events=evs[i] if evs is not None else None)
@@ -258,7 +262,7 @@ def main():
     orient_before = list(orient)
     t_start.record()
     for s in range(args.steps):
-        one_step(evs[s] if "batch" not in wl else None)
+        one_step(evs[s] if ("batch" not in wl and args.algo == "3stage") else None)
     t_end.record()
     torch.cuda.synchronize()
     launches = ipt.kernel_launch_count() - launches0
@@ -285,7 +289,7 @@ def main():
     kern_n = {"cycle_global": 0, "tile_onchip": 0}
     stage_scaled = None
     per_shape = {}
-    if "batch" not in wl:
+    if "batch" not in wl and args.algo == "3stage":
         orient_sim = list(orient_before)
         S_bytes = 0
         for s in range(args.steps):
@@ -421,7 +425,8 @@ def main():
                        "elem_bytes": eb, "batch": wl.get("batch", 1),
                        "plans": plans_cfg,
                        "l2": "no flush: every matrix exceeds the 126 MB L2" if args.workload in ("sweep", "c3", "c4", "c5") else "L2-resident (52 MB)",
-                       "parallelism": f"replicas x{world}" if "batch" not in wl else f"batch shards x{world}"},
+                       "parallelism": f"replicas x{world}" if "batch" not in wl else f"batch shards x{world}",
+                       "algo": args.algo},
             "hbm_frac_stage_scaled": round(stage_scaled, 4) if stage_scaled else None,
             "per_shape": per_shape, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
             "clocks": clk, "verified": ok,

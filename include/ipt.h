@@ -125,6 +125,14 @@ ipt_status ipt_transpose_batched_plan(void *d_base, int64_t count, int64_t strid
                                       const ipt_plan_t *plan, void *d_workspace,
                                       size_t ws_bytes, void *stream);
 
+/* The paper's 4-stage Gustavson/Karlsson baseline (Fig. 2): 0100!, 0010!, 1000!,
+ * 0100! on the 4-D view M' x m x N' x n, with the same kernels.  m | M, n | N, or 0 to
+ * take the 3-stage planner's tiles.  Kept to reproduce the paper's 3-stage vs 4-stage
+ * comparison (Table 2); same conventions as ipt_transpose_plan. */
+ipt_status ipt_transpose_4stage(void *d_ptr, int64_t M, int64_t N, int64_t m, int64_t n,
+                                int elem_bytes, void *d_workspace, size_t ws_bytes,
+                                void *stream);
+
 /* ----------------------------------------------- host-delegated transposition (Sec. 6) */
 
 /* In-place transposition of a HOST array executed on the GPU (Fig. 4/5):

@@ -67,6 +67,7 @@ ABI = [
     ("ipt_transpose_plan_events", _int, [_vp, ctypes.POINTER(Plan), _vp, _sz, _vp, ctypes.POINTER(_vp)]),
     ("ipt_transpose_batched", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp]),
     ("ipt_transpose_batched_plan", _int, [_vp, _i64, _i64, ctypes.POINTER(Plan), _vp, _sz, _vp]),
+    ("ipt_transpose_4stage", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
     ("ipt_transpose_host", _int, [_vp, _i64, _i64, _int, _int, _vp, _sz, _vp]),
     ("ipt_stage_workspace_bytes", _sz, [_i64, _i64, _i64, _i64, _int]),
     ("ipt_100", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
@@ -196,6 +197,17 @@ def transpose_batched_(t, count: int, M: int, N: int, stride_elems: int | None =
         _check(lib().ipt_transpose_batched_plan(ptr, count, stride, ctypes.byref(plan_), None, 0, st),
                "ipt_transpose_batched_plan")
     return t
+
+
+def transpose_4stage_(t, M: int, N: int, m: int = 0, n: int = 0, stream=None,
+                      elem_bytes: int | None = None):
+    """The paper's 4-stage Gustavson/Karlsson baseline on the GPU, in place."""
+    eb = _eb(t, elem_bytes)
+    if _nelem(t, eb) != M * N:
+        raise IptError(f"elements {_nelem(t, eb)} != M*N {M * N}")
+    _check(lib().ipt_transpose_4stage(_dev_ptr(t), M, N, m, n, eb, None, 0, _stream_ptr(stream)),
+           "ipt_transpose_4stage")
+    return t.view(N, M) if eb == t.element_size() else t
 
 
 def transpose_host_(h, M: int, N: int, queues: int = 4, stream=None, elem_bytes: int | None = None):

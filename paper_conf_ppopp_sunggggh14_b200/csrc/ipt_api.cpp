@@ -413,6 +413,64 @@ ipt_status ipt_1000(void *d_ptr, int64_t d0, int64_t d1, int64_t d2, int64_t d3,
     return ipt_100(d_ptr, 1, d0, d1, s, elem_bytes, d_workspace, ws_bytes, stream);
 }
 
+// ---------------------------------------------- 4-stage baseline (Fig. 2; NEXT-2)
+// Gustavson/Karlsson 4-stage sequence on the 4-D view M' x m x N' x n:
+//   0100!  P(M', m, N', n)     M' instances of m x N' with n-element super-elements
+//   0010!  P(M'N', m, n, 1)    every m x n tile
+//   1000!  P(1, M', N', m*n)   one M' x N' array of (m*n)-element super-elements
+//   0100!  P(N', M', n, m)     N' instances of M' x n with m-element super-elements
+// Same kernels as the 3-stage path; kept as the paper's baseline for its 3x claim (Table 2).
+ipt_status ipt_transpose_4stage(void *d_ptr, int64_t M, int64_t N, int64_t m, int64_t n,
+                                int elem_bytes, void *d_workspace, size_t ws_bytes,
+                                void *stream) {
+    ipt_status s = check_shape(M, N, elem_bytes, nullptr);
+    if (s) return s;
+    if ((s = check_ptr(d_ptr, elem_bytes))) return s;
+    if (m < 0 || n < 0 || (m && M % m) || (n && N % n)) return IPT_ERR_INVALID_ARG;
+    if (M == 1 || N == 1) return IPT_OK;
+    const int device = current_device();
+    if (device < 0) return IPT_ERR_NO_DEVICE;
+    if (!m || !n) {
+        ipt_plan_t p;
+        if ((s = ipt_plan(M, N, elem_bytes, device, &p))) return s;
+        if (!m) m = p.m;
+        if (!n) n = p.n;
+    }
+    const int64_t Mp = M / m, Np = N / n;
+    StageDesc sd[4];
+    for (int i = 0; i < 4; ++i) {
+        sd[i] = StageDesc{};
+        sd[i].base = (char *)d_ptr;
+        sd[i].inner = 1;
+        sd[i].eb = elem_bytes;
+    }
+    sd[0].outer = Mp;      sd[0].A = m;  sd[0].B = Np; sd[0].s = n;
+    sd[1].outer = Mp * Np; sd[1].A = m;  sd[1].B = n;  sd[1].s = 1;
+    sd[2].outer = 1;       sd[2].A = Mp; sd[2].B = Np; sd[2].s = m * n;
+    sd[3].outer = Np;      sd[3].A = Mp; sd[3].B = n;  sd[3].s = m;
+    size_t need = 0;
+    bool tile2 = false;
+    for (int i = 0; i < 4; ++i) {
+        sd[i].ostride = sd[i].A * sd[i].B * sd[i].s * elem_bytes;
+        if (sd[i].A == 1 || sd[i].B == 1) continue;
+        if (i == 1 && tile_onchip_fits(m, n, elem_bytes, device)) { tile2 = true; continue; }
+        need = std::max(need, cycle_ws_bytes(sd[i]));
+    }
+    void *ws = d_workspace;
+    if (!ws) {
+        if ((s = get_ws(device, stream, need, &ws))) return s;
+    } else if (ws_bytes < need) {
+        return IPT_ERR_NO_MEMORY;
+    }
+    for (int i = 0; i < 4; ++i) {
+        if (sd[i].A == 1 || sd[i].B == 1) continue;
+        cudaError_t e = (i == 1 && tile2) ? launch_tile_onchip(sd[i], (cudaStream_t)stream, device)
+                                          : launch_cycle_global(sd[i], ws, (cudaStream_t)stream, device);
+        if (e != cudaSuccess) return cuda_status(e);
+    }
+    return IPT_OK;
+}
+
 // ------------------------------------------------- host-delegated transposition (Sec. 6)
 // the matrix is copied to the GPU (1), transposed in place there (2), and
 // copied back to the same host location (3).  Stage 1 (100!) spans the whole array and

@@ -431,3 +431,16 @@ def test_ipt_010_generic_cluster_column_split(monkeypatch, eb, batch, A, B):
     t = to_dev(a, eb)
     ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
     assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)
+
+
+# ------------------------------------------------ 4-stage baseline (NEXT-2)
+@pytest.mark.parametrize("M,N,m,n", [(120, 72, 8, 6), (360, 1000, 40, 25), (97, 64, 97, 8),
+                                     (1800, 720, 0, 0), (256, 256, 16, 16)])
+def test_4stage_matches_oracle(M, N, m, n):
+    a = seeded.matrix_np(M, N, 4)
+    t = to_dev(a, 4)
+    ipt.transpose_4stage_(t, M, N, m, n)
+    ref = oracle.transpose_inplace(a.copy(), M, N)
+    assert np.array_equal(to_np(t, 4), ref)
+    if m and n:   # and stage by stage equal to the oracle's own 4-stage composition
+        assert np.array_equal(ref, oracle.transpose_4stage(a.copy(), M, N, m, n))

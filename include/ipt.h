@@ -175,6 +175,20 @@ ipt_status ipt_0100(void *d_ptr, int64_t d0, int64_t d1, int64_t d2, int64_t d3,
 ipt_status ipt_1000(void *d_ptr, int64_t d0, int64_t d1, int64_t d2, int64_t d3,
                     int elem_bytes, void *d_workspace, size_t ws_bytes, void *stream);
 
+/* ------------------------------------ layout marshaling (Sung et al.'s DL system) */
+/* AoS: M structures of N fields (row-major M x N).  SoA: N x M.  ASTA (Array of Structures
+ * of Tiled Arrays) with tiles of m structures (m | M): M/m x N x m.  AoS -> ASTA is 010!
+ * on (M/m) x m x N; SoA -> ASTA is 100! on N x (M/m) x m.  The *_to_aos / *_to_soa
+ * calls are the inverse transformations.  Same conventions as ipt_010 / ipt_100. */
+ipt_status ipt_aos_to_asta(void *d_ptr, int64_t M, int64_t N, int64_t m, int elem_bytes,
+                           void *d_workspace, size_t ws_bytes, void *stream);
+ipt_status ipt_asta_to_aos(void *d_ptr, int64_t M, int64_t N, int64_t m, int elem_bytes,
+                           void *d_workspace, size_t ws_bytes, void *stream);
+ipt_status ipt_soa_to_asta(void *d_ptr, int64_t M, int64_t N, int64_t m, int elem_bytes,
+                           void *d_workspace, size_t ws_bytes, void *stream);
+ipt_status ipt_asta_to_soa(void *d_ptr, int64_t M, int64_t N, int64_t m, int elem_bytes,
+                           void *d_workspace, size_t ws_bytes, void *stream);
+
 /* ------------------------------------------------------------------- diagnostics */
 
 const char *ipt_status_string(ipt_status s);

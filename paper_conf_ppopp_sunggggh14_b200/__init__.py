@@ -75,6 +75,10 @@ ABI = [
     ("ipt_0010", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
     ("ipt_0100", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
     ("ipt_1000", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
+    ("ipt_aos_to_asta", _int, [_vp, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
+    ("ipt_asta_to_aos", _int, [_vp, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
+    ("ipt_soa_to_asta", _int, [_vp, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
+    ("ipt_asta_to_soa", _int, [_vp, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
     ("ipt_status_string", ctypes.c_char_p, [_int]),
     ("ipt_kernel_launch_count", ctypes.c_uint64, []),
     ("ipt_last_cuda_error", ctypes.c_char_p, []),
@@ -253,6 +257,25 @@ def ipt_1000_(t, d0: int, d1: int, d2: int, d3: int, stream=None, elem_bytes: in
     _check(lib().ipt_1000(_dev_ptr(t), d0, d1, d2, d3, _eb(t, elem_bytes), None, 0,
                           _stream_ptr(stream)), "ipt_1000")
     return t
+
+
+# ------------------------------------------------ layout marshaling (NEXT-3)
+def _marshal(name):
+    def f(t, M: int, N: int, m: int, stream=None, elem_bytes: int | None = None):
+        eb = _eb(t, elem_bytes)
+        if _nelem(t, eb) != M * N:
+            raise IptError(f"elements {_nelem(t, eb)} != M*N {M * N}")
+        _check(getattr(lib(), name)(_dev_ptr(t), M, N, m, eb, None, 0, _stream_ptr(stream)), name)
+        return t
+    f.__name__ = name[4:] + "_"
+    f.__doc__ = (f"{name}: M structures x N fields, tiles of m structures (P:140); in place.")
+    return f
+
+
+aos_to_asta_ = _marshal("ipt_aos_to_asta")
+asta_to_aos_ = _marshal("ipt_asta_to_aos")
+soa_to_asta_ = _marshal("ipt_soa_to_asta")
+asta_to_soa_ = _marshal("ipt_asta_to_soa")
 
 
 def kernel_launch_count() -> int:

@@ -583,6 +583,35 @@ ipt_status ipt_transpose_host(void *h_ptr, int64_t M, int64_t N, int elem_bytes,
     return cuda_status(e);
 }
 
+// ------------------------------------------- layout marshaling (Sung's DL; NEXT-3)
+// Array-of-Structures / Structure-of-Arrays <-> Array-of-Structures-of-Tiled-Arrays.
+// AoS = M structures x N fields; ASTA groups the structures in tiles of m (M = M' m):
+// M' x N x m.  AoS -> ASTA is 010! on M' x m x N; SoA (N x M' x m) -> ASTA is 100!
+// (P:140).  The inverse transformations are the inverse elementary transpositions.
+ipt_status ipt_aos_to_asta(void *d_ptr, int64_t M, int64_t N, int64_t m, int elem_bytes,
+                           void *d_workspace, size_t ws_bytes, void *stream) {
+    if (m < 1 || M < 1 || M % m) return IPT_ERR_INVALID_ARG;
+    return ipt_010(d_ptr, M / m, m, N, elem_bytes, d_workspace, ws_bytes, stream);
+}
+
+ipt_status ipt_asta_to_aos(void *d_ptr, int64_t M, int64_t N, int64_t m, int elem_bytes,
+                           void *d_workspace, size_t ws_bytes, void *stream) {
+    if (m < 1 || M < 1 || M % m) return IPT_ERR_INVALID_ARG;
+    return ipt_010(d_ptr, M / m, N, m, elem_bytes, d_workspace, ws_bytes, stream);
+}
+
+ipt_status ipt_soa_to_asta(void *d_ptr, int64_t M, int64_t N, int64_t m, int elem_bytes,
+                           void *d_workspace, size_t ws_bytes, void *stream) {
+    if (m < 1 || M < 1 || M % m) return IPT_ERR_INVALID_ARG;
+    return ipt_100(d_ptr, 1, N, M / m, m, elem_bytes, d_workspace, ws_bytes, stream);
+}
+
+ipt_status ipt_asta_to_soa(void *d_ptr, int64_t M, int64_t N, int64_t m, int elem_bytes,
+                           void *d_workspace, size_t ws_bytes, void *stream) {
+    if (m < 1 || M < 1 || M % m) return IPT_ERR_INVALID_ARG;
+    return ipt_100(d_ptr, 1, M / m, N, m, elem_bytes, d_workspace, ws_bytes, stream);
+}
+
 // -------------------------------------------------------------------- diagnostics
 const char *ipt_status_string(ipt_status s) {
     switch (s) {

@@ -444,3 +444,26 @@ def test_4stage_matches_oracle(M, N, m, n):
     assert np.array_equal(to_np(t, 4), ref)
     if m and n:   # and stage by stage equal to the oracle's own 4-stage composition
         assert np.array_equal(ref, oracle.transpose_4stage(a.copy(), M, N, m, n))
+
+
+# ---------------------------------------- layout marshaling AoS/SoA <-> ASTA (NEXT-3)
+@pytest.mark.parametrize("M,N,m", [(1000, 256, 100), (4096, 64, 32), (999, 7, 37), (1_000_000, 256, 64)])
+def test_layout_marshaling(M, N, m):
+    """AoS (M x N) -> ASTA (M/m x N x m) = 010!; SoA (N x M) -> ASTA = 100!; and
+    their inverses.  K-Means descriptor shape included (1e6 x 256)."""
+    Mp = M // m
+    a = seeded.matrix_np(M, N, 4)
+    asta = a.reshape(Mp, m, N).transpose(0, 2, 1).reshape(-1)
+    t = to_dev(a, 4)
+    ipt.aos_to_asta_(t, M, N, m)
+    if M * N <= 4_000_000:
+        assert np.array_equal(to_np(t, 4), oracle.permute_inplace(a.copy(), Mp, m, N, 1))
+    assert np.array_equal(to_np(t, 4), asta)
+    ipt.asta_to_aos_(t, M, N, m)
+    assert np.array_equal(to_np(t, 4), a)
+    soa = a.reshape(M, N).T.reshape(-1).copy()
+    t = to_dev(soa, 4)
+    ipt.soa_to_asta_(t, M, N, m)
+    assert np.array_equal(to_np(t, 4), asta)
+    ipt.asta_to_soa_(t, M, N, m)
+    assert np.array_equal(to_np(t, 4), soa)

@@ -219,6 +219,18 @@ __global__ void __launch_bounds__(512, 2) tile_onchip_ldg(const TileParams p) {
     }
 }
 
+__device__ __forceinline__ FastDiv32 make_fastdiv32_dev(uint32_t d) {
+    FastDiv32 f;
+    if (d == 0) d = 1;
+    f.d = d;
+    const uint32_t l = (d > 1) ? 32 - __clz(d - 1) : 0;
+    const uint64_t two_l = (uint64_t)1 << l;
+    f.m = (uint32_t)((((two_l - d) << 32) / d) + 1);
+    f.s1 = l ? 1 : 0;
+    f.s2 = l ? l - 1 : 0;
+    return f;
+}
+
 // -------------------------------------------------------------- cluster-split kernel
 // Tiles larger than one CTA's shared memory: a thread-block cluster of K CTAs (K SMs)
 // owns one tile; CTA k holds tile rows [k*m/K, (k+1)*m/K) and writes exactly the output
@@ -245,10 +257,14 @@ __global__ void __launch_bounds__(512, 2) tile_onchip_cluster(const TileParams p
     const uint32_t K = p.K;
     const uint32_t rank = cluster_rank();
     const uint32_t cid = blockIdx.x / K, ncl = gridDim.x / K;
-    const uint32_t rows = p.m / K;                 // tile rows held by this CTA
+    const uint32_t mv = p.m / V;                   // V-row blocks, split (unevenly) over K
+    const uint32_t b0 = (uint32_t)((uint64_t)rank * mv / K);
+    const uint32_t b1 = (uint32_t)((uint64_t)(rank + 1) * mv / K);
+    const uint32_t rows = (b1 - b0) * V;           // tile rows held by this CTA
     const uint32_t nvrow = p.n / V;                // 16-byte vectors per row
     const uint32_t nvec = rows * nvrow;
-    const size_t slice_off = (size_t)rank * rows * p.n * EB;
+    const size_t slice_off = (size_t)b0 * V * p.n * EB;
+    const FastDiv32 divmvp = make_fastdiv32_dev(b1 - b0);
     for (uint64_t t = cid; t < p.count; t += ncl) {
         char *g = tile_ptr(p, t);
         const char *src = g + slice_off;
@@ -270,7 +286,7 @@ __global__ void __launch_bounds__(512, 2) tile_onchip_cluster(const TileParams p
             }
         }
         cluster_sync_all();     // every slice of tile t is on chip before anyone stores
-        write_out<EB>(p, sbase, g, rank * (rows / V), rows / V, p.divMVK32);
+        write_out<EB>(p, sbase, g, b0, b1 - b0, divmvp);
         __syncthreads();        // shared slice consumed before the next tile's loads
     }
 }
@@ -375,17 +391,6 @@ __global__ void __launch_bounds__(512) tile_onchip_generic(const TileParams p) {
 // K-CTA cluster holds rows [k*m/K, (k+1)*m/K) (uneven slices allowed) and writes the
 // matching column segment of every output row with coalesced element stores.  One
 // cluster barrier per tile separates all loads of the tile from all stores into it.
-__device__ __forceinline__ FastDiv32 make_fastdiv32_dev(uint32_t d) {
-    FastDiv32 f;
-    if (d == 0) d = 1;
-    f.d = d;
-    const uint32_t l = (d > 1) ? 32 - __clz(d - 1) : 0;
-    const uint64_t two_l = (uint64_t)1 << l;
-    f.m = (uint32_t)((((two_l - d) << 32) / d) + 1);
-    f.s1 = l ? 1 : 0;
-    f.s2 = l ? l - 1 : 0;
-    return f;
-}
 
 template <typename T>
 __global__ void __launch_bounds__(512, 1) tile_generic_cluster(const TileParams p) {
@@ -593,8 +598,8 @@ int tile_cluster_k(int64_t A, int64_t B, int eb, int device) {
     const size_t rowb = (size_t)fast_q(B, eb) * 16;
     int fit = 0;
     for (int K : {2, 4, 8}) {
-        if (A % (K * V)) continue;
-        const size_t slice = (size_t)(A / K) * rowb;
+        if (A / V < K) break;
+        const size_t slice = (size_t)((A / V + K - 1) / K) * V * rowb;   // largest slice
         if (slice <= 113 * 1024) return K;
         if (!fit && (long)slice <= budget) fit = K;
     }
@@ -686,7 +691,7 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
             p.K = (uint32_t)K;
             p.divMVK32 = make_fastdiv32((uint32_t)(d.A / V / K));
             p.divNV32 = make_fastdiv32((uint32_t)(d.B / V));
-            const size_t smem = (size_t)(d.A / K) * p.q * 16;
+            const size_t smem = (size_t)((d.A / V + K - 1) / K) * V * p.q * 16;
             switch (d.eb) {
                 case 4: return go_cluster(tile_onchip_cluster<4, 8>, p, smem, K, st, device);
                 case 8: return go_cluster(tile_onchip_cluster<8, 8>, p, smem, K, st, device);

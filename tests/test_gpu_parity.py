@@ -467,3 +467,12 @@ def test_layout_marshaling(M, N, m):
     assert np.array_equal(to_np(t, 4), asta)
     ipt.asta_to_soa_(t, M, N, m)
     assert np.array_equal(to_np(t, 4), soa)
+
+
+@pytest.mark.parametrize("eb,batch,A,B", [(4, 2, 1800, 240), (8, 3, 902, 100), (4, 2, 3004, 128)])
+def test_ipt_010_cluster_uneven_slices(eb, batch, A, B):
+    """16-byte cluster path with row slices of unequal length (multiples of V rows)."""
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)

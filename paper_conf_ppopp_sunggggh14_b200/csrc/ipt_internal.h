@@ -91,6 +91,7 @@ bool tile_onchip_fits(int64_t A, int64_t B, int eb, int device);
 // 4: element path split over a thread-block cluster
 int tile_onchip_path(int64_t A, int64_t B, int eb, int device);
 int tile_cluster_k(int64_t A, int64_t B, int eb, int device);
+int tile_generic_cluster_k(int64_t A, int64_t B, int eb, int device);
 cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device);
 
 // Device properties used by planner and launchers (cached).

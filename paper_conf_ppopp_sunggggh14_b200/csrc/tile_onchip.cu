@@ -103,27 +103,28 @@ __device__ __forceinline__ void sts128(uint32_t saddr, const uint4 &v) {
                  :: "r"(saddr), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
 }
 
-// Write the transposed tile from padded shared memory (sbase, pitch q) to global g.
-// Only block rows [bi0, bi0 + mvp) of the tile (in V-row units) are in this CTA's shared
-// memory (row bil*V of the buffer holds tile row (bi0 + bil)*V): the whole tile for the
-// single-CTA kernels, one slice for the cluster kernel.
+// Write the transposed tile from padded shared memory to global g.  The CTA holds the
+// block rows [bi0, bi0 + mvp) x block columns [bj0, bj0 + nbj) of the tile (V x V blocks):
+// buffer row bil*V + r, 16-byte column bjl (pitch q) holds tile row (bi0+bil)*V + r,
+// columns (bj0+bjl)*V .. +V-1.  Whole tile for one CTA; a row or column slice per cluster CTA.
 template <int EB>
-__device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, char *g,
-                                          uint32_t bi0, uint32_t mvp, const FastDiv32 &divmvp) {
+__device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, char *g, uint32_t q,
+                                          uint32_t bi0, uint32_t mvp, const FastDiv32 &divmvp,
+                                          uint32_t bj0, uint32_t nbj) {
     constexpr int V = 16 / EB;
     constexpr int ROT = (V >= 8) ? 1 : 8 / V;   // lanes sharing one rotation
     using E = typename Elem<EB>::T;
-    const uint32_t nblk = mvp * (p.n / V);
+    const uint32_t nblk = mvp * nbj;
     for (uint32_t blk = threadIdx.x; blk < nblk; blk += blockDim.x) {
-        uint32_t bj, bil;
-        fdivmod32(blk, divmvp, bj, bil);
-        const uint32_t bi = bi0 + bil;
+        uint32_t bjl, bil;
+        fdivmod32(blk, divmvp, bjl, bil);
+        const uint32_t bi = bi0 + bil, bj = bj0 + bjl;
         const int off = (int)((bil / ROT) % V);
         E x[V][V];
 #pragma unroll
         for (int kk = 0; kk < V; ++kk) {
             const uint32_t rho = (uint32_t)((kk + off) % V);
-            const uint4 v = lds128(sbase + ((bil * V + rho) * p.q + bj) * 16);
+            const uint4 v = lds128(sbase + ((bil * V + rho) * q + bjl) * 16);
             unpack<EB>(v, x[kk]);
         }
         // x[kk][c] = tile[bi*V + (kk+off)%V][bj*V + c]; output row bj*V+c gets column c.
@@ -140,7 +141,7 @@ __device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, c
 
 template <int EB>
 __device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, char *g) {
-    write_out<EB>(p, sbase, g, 0, p.m / (16 / EB), p.divMV32);
+    write_out<EB>(p, sbase, g, p.q, 0, p.m / (16 / EB), p.divMV32, 0, p.n / (16 / EB));
 }
 
 // ------------------------------------------------------------------- TMA ring kernel
@@ -257,36 +258,48 @@ __global__ void __launch_bounds__(512, 2) tile_onchip_cluster(const TileParams p
     const uint32_t K = p.K;
     const uint32_t rank = cluster_rank();
     const uint32_t cid = blockIdx.x / K, ncl = gridDim.x / K;
-    const uint32_t mv = p.m / V;                   // V-row blocks, split (unevenly) over K
-    const uint32_t b0 = (uint32_t)((uint64_t)rank * mv / K);
-    const uint32_t b1 = (uint32_t)((uint64_t)(rank + 1) * mv / K);
-    const uint32_t rows = (b1 - b0) * V;           // tile rows held by this CTA
-    const uint32_t nvrow = p.n / V;                // 16-byte vectors per row
-    const uint32_t nvec = rows * nvrow;
-    const size_t slice_off = (size_t)b0 * V * p.n * EB;
+    const uint32_t mv = p.m / V, nvr = p.n / V;    // V-row blocks, 16-byte vectors per row
+    uint32_t b0, b1, c0, c1, q;
+    if (!p.colsplit) {   // rows [b0, b1) (V-row blocks), all columns
+        b0 = (uint32_t)((uint64_t)rank * mv / K);
+        b1 = (uint32_t)((uint64_t)(rank + 1) * mv / K);
+        c0 = 0; c1 = nvr; q = p.q;
+    } else {             // all rows, 16-byte columns [c0, c1) (one vector = V columns)
+        b0 = 0; b1 = mv;
+        c0 = (uint32_t)((uint64_t)rank * nvr / K);
+        c1 = (uint32_t)((uint64_t)(rank + 1) * nvr / K);
+        q = (c1 - c0) | 1u;
+    }
+    const uint32_t rows = (b1 - b0) * V, cvec = c1 - c0;
+    const uint32_t nvec = rows * cvec;
     const FastDiv32 divmvp = make_fastdiv32_dev(b1 - b0);
+    const FastDiv32 divc = make_fastdiv32_dev(cvec);
     for (uint64_t t = cid; t < p.count; t += ncl) {
         char *g = tile_ptr(p, t);
-        const char *src = g + slice_off;
+        const char *src = g + ((size_t)b0 * V * nvr + c0) * 16;
         for (uint32_t e0 = threadIdx.x; e0 < nvec; e0 += U * blockDim.x) {
             uint4 v[U];
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const uint32_t e = e0 + u * blockDim.x;
-                if (e < nvec) v[u] = ld_cg<16>(src + (size_t)e * 16);
+                if (e < nvec) {
+                    uint32_t i, j;
+                    fdivmod32(e, divc, i, j);
+                    v[u] = ld_cg<16>(src + ((size_t)i * nvr + j) * 16);
+                }
             }
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const uint32_t e = e0 + u * blockDim.x;
                 if (e < nvec) {
                     uint32_t i, j;
-                    fdivmod32(e, p.divNV32, i, j);
-                    sts128(sbase + (i * p.q + j) * 16, v[u]);
+                    fdivmod32(e, divc, i, j);
+                    sts128(sbase + (i * q + j) * 16, v[u]);
                 }
             }
         }
         cluster_sync_all();     // every slice of tile t is on chip before anyone stores
-        write_out<EB>(p, sbase, g, b0, b1 - b0, divmvp);
+        write_out<EB>(p, sbase, g, q, b0, b1 - b0, divmvp, c0, cvec);
         __syncthreads();        // shared slice consumed before the next tile's loads
     }
 }
@@ -590,16 +603,30 @@ cudaError_t go_cluster(K_ kern, const TileParams &p, size_t smem, int K, cudaStr
 
 // Cluster size for a tile that does not fit one CTA (0 = none): the smallest K in
 // {2, 4, 8} whose row slice fits 113 KB (two CTAs per SM), else the smallest that fits.
+// Fast-path cluster split: column split when the tile has fewer rows than columns (each
+// CTA then writes whole contiguous output rows), else row split.
+static bool fast_colsplit(int64_t A, int64_t B, int eb) {
+    // row-split write segments are ~A*eb/K bytes: only short rows (< 1 KB) favour columns
+    return A < B && A * eb < 1024 && env_int("IPT_TILE_FAST_COLSPLIT", 1);
+}
+
 int tile_cluster_k(int64_t A, int64_t B, int eb, int device) {
     if (!vec_ok(A, B, eb) || !env_int("IPT_TILE_CLUSTER", 1)) return 0;
     DevProps dp = dev_props(device);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
     const int V = 16 / eb;
-    const size_t rowb = (size_t)fast_q(B, eb) * 16;
+    const bool cs = fast_colsplit(A, B, eb);
     int fit = 0;
-    for (int K : {2, 4, 8}) {
-        if (A / V < K) break;
-        const size_t slice = (size_t)((A / V + K - 1) / K) * V * rowb;   // largest slice
+    for (int K : {2, 4, 8, 16}) {
+        size_t slice;
+        if (cs) {
+            const int64_t nvr = B / V;
+            if (nvr < K) break;
+            slice = (size_t)A * (size_t)(((nvr + K - 1) / K) | 1) * 16;
+        } else {
+            if (A / V < K) break;
+            slice = (size_t)((A / V + K - 1) / K) * V * (size_t)fast_q(B, eb) * 16;
+        }
         if (slice <= 113 * 1024) return K;
         if (!fit && (long)slice <= budget) fit = K;
     }
@@ -618,7 +645,7 @@ int tile_generic_cluster_k(int64_t A, int64_t B, int eb, int device) {
     DevProps dp = dev_props(device);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
     const bool cs = generic_colsplit(A, B);
-    for (int K : {2, 4, 8}) {
+    for (int K : {2, 4, 8, 16}) {
         size_t bytes;
         if (cs) {
             if (B < K) break;
@@ -689,9 +716,11 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
             const int V = 16 / d.eb;
             p.q = fast_q(d.B, d.eb);
             p.K = (uint32_t)K;
-            p.divMVK32 = make_fastdiv32((uint32_t)(d.A / V / K));
-            p.divNV32 = make_fastdiv32((uint32_t)(d.B / V));
-            const size_t smem = (size_t)((d.A / V + K - 1) / K) * V * p.q * 16;
+            p.colsplit = fast_colsplit(d.A, d.B, d.eb) ? 1 : 0;
+            const int64_t nvr = d.B / V;
+            const size_t smem = p.colsplit
+                ? (size_t)d.A * (size_t)(((nvr + K - 1) / K) | 1) * 16
+                : (size_t)((d.A / V + K - 1) / K) * V * p.q * 16;
             switch (d.eb) {
                 case 4: return go_cluster(tile_onchip_cluster<4, 8>, p, smem, K, st, device);
                 case 8: return go_cluster(tile_onchip_cluster<8, 8>, p, smem, K, st, device);

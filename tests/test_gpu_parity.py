@@ -476,3 +476,23 @@ def test_ipt_010_cluster_uneven_slices(eb, batch, A, B):
     t = to_dev(a, eb)
     ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
     assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)
+
+
+@pytest.mark.parametrize("eb,batch,A,B", [(4, 2, 7200, 120), (4, 1, 9998, 64)])
+def test_ipt_010_cluster16(eb, batch, A, B):
+    """Non-portable 16-CTA clusters (panels up to 16 x 227 KB)."""
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)
+
+
+@pytest.mark.parametrize("eb,batch,A,B", [(4, 2, 120, 7200), (8, 2, 64, 2000), (16, 2, 32, 3000),
+                                          (4, 3, 256, 1000)])
+def test_ipt_010_cluster_column_split_fast(eb, batch, A, B):
+    """16-byte cluster path, fewer rows than columns: each CTA owns a range of 16-byte
+    columns and writes whole contiguous output rows."""
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)

@@ -66,6 +66,8 @@ struct CycParams {
     uint64_t units;     // batch * A*B * nchunk
     uint64_t nwords;    // flag words
     uint64_t wstride;   // start-order scramble (coprime to nwords)
+    uint64_t nfetch;    // fetches = nwords << segsh (a fetch is a segment of a flag word)
+    uint32_t segsh;     // log2(segments per flag word): small stages hand out fewer units
     Div2 divB, divAB, divInner, divNchunk, divNwords;
     uint32_t *flags;
     unsigned long long *counter;
@@ -118,14 +120,18 @@ cycle_global_kernel(const CycParams p) {
                 unsigned long long wb = 0;
                 if (lane == leader) wb = atomicAdd(p.counter, (unsigned long long)__popc(need));
                 wb = __shfl_sync(FULL, wb, leader);
-                uint64_t mine64 = wb + __popc(need & ((1u << g0) - 1u));
-                const bool have = mine64 < p.nwords;
+                const uint64_t f = wb + __popc(need & ((1u << g0) - 1u));
+                const bool have = f < p.nfetch;
+                const uint64_t mine64 = f >> p.segsh;
+                const uint32_t seg = (uint32_t)(f & ((1u << p.segsh) - 1u));
                 I mine = (I)mine64;
                 if (have && p.wstride != 1) {
                     uint64_t q, r;
                     fdivmod(mine64 * p.wstride, p.divNwords.d64, q, r);
                     mine = (I)r;
                 }
+                const uint32_t F = 32u >> p.segsh;
+                const uint32_t segmask = (F == 32) ? 0xffffffffu : (((1u << F) - 1u) << (seg * F));
                 uint32_t fw = 0;
                 if (mode == M_FETCH && have) fw = ld_relaxed_u32(p.flags + mine);
                 fw = __shfl_sync(FULL, fw, g0);
@@ -134,7 +140,7 @@ cycle_global_kernel(const CycParams p) {
                     if (!have) {
                         mode = M_DONE;
                     } else {
-                        cw = fw;
+                        cw = fw | ~segmask;     // bits outside this segment: not ours
                         nb = 0;
                         mode = M_SCAN;
                     }
@@ -315,15 +321,18 @@ __global__ void __launch_bounds__(256, 6) cycle_ua_kernel(const CycParams p) {
                 unsigned long long wb = 0;
                 if (lane == 0) wb = atomicAdd(p.counter, 1ull);
                 wb = __shfl_sync(FULL, wb, 0);
-                if (wb >= p.nwords) { mode = M_DONE; break; }
-                uint64_t mine = wb;
+                if (wb >= p.nfetch) { mode = M_DONE; break; }
+                uint64_t mine = wb >> p.segsh;
+                const uint32_t seg = (uint32_t)(wb & ((1u << p.segsh) - 1u));
                 if (p.wstride != 1) {
                     uint64_t q, r;
-                    fdivmod(wb * p.wstride, p.divNwords.d64, q, r);
+                    fdivmod(mine * p.wstride, p.divNwords.d64, q, r);
                     mine = r;
                 }
                 word = (I)mine;
-                cw = ld_relaxed_u32(p.flags + word);
+                const uint32_t F = 32u >> p.segsh;
+                const uint32_t segmask = (F == 32) ? 0xffffffffu : (((1u << F) - 1u) << (seg * F));
+                cw = ld_relaxed_u32(p.flags + word) | ~segmask;
                 cw = __shfl_sync(FULL, cw, 0);
                 nb = 0;
                 mode = M_SCAN;
@@ -534,7 +543,7 @@ cudaError_t launch_t(const CycParams &p, cudaStream_t st, int device) {
     if (occ_cap > 0 && occ_cap < per_sm) per_sm = (int)occ_cap;
     uint64_t grid = (uint64_t)dp.sms * (uint64_t)(per_sm > 0 ? per_sm : 1);
     const uint64_t groups_per_block = 8ull * (32 / G);
-    const uint64_t need = (p.nwords + groups_per_block - 1) / groups_per_block;
+    const uint64_t need = (p.nfetch + groups_per_block - 1) / groups_per_block;
     if (need < grid) grid = need;
     if (grid < 1) grid = 1;
     kern<<<(unsigned)grid, 256, 0, st>>>(p);
@@ -561,7 +570,7 @@ cudaError_t launch_ua(const CycParams &p, cudaStream_t st, int device) {
     }
     DevProps dp = dev_props(device);
     uint64_t grid = (uint64_t)dp.sms * (uint64_t)(per_sm > 0 ? per_sm : 1);
-    const uint64_t need = (p.nwords + 7) / 8;
+    const uint64_t need = (p.nfetch + 7) / 8;
     if (need < grid) grid = need;
     if (grid < 1) grid = 1;
     kern<<<(unsigned)grid, 256, 0, st>>>(p);
@@ -640,6 +649,18 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
     p.cvec = c.cvec;
     p.units = units;
     p.nwords = (p.units + 31) / 32;
+    {
+        // Small stages: hand out segments of a flag word so that every resident walker
+        // gets a start (parallelism = fetches, not words).
+        const DevProps dp = dev_props(device);
+        const uint64_t walkers = (uint64_t)dp.sms * 64 * (c.ua ? 1 : (32 / c.G));
+        long forced = env_int("IPT_CYC_SEGSH", -1);
+        uint32_t sh = 0;
+        while (sh < 5 && (p.nwords << sh) < 2 * walkers) ++sh;
+        if (forced >= 0 && forced <= 5) sh = (uint32_t)forced;
+        p.segsh = sh;
+        p.nfetch = p.nwords << sh;
+    }
     p.wstride = 1;
     {
         const uint64_t batch = (uint64_t)d.outer * d.inner;

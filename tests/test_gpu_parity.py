@@ -496,3 +496,14 @@ def test_ipt_010_cluster_column_split_fast(eb, batch, A, B):
     t = to_dev(a, eb)
     ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
     assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)
+
+
+@pytest.mark.parametrize("segsh", [0, 2, 5])
+def test_ipt_100_fetch_segments(monkeypatch, segsh):
+    """Start units handed out as 1/2^segsh of a flag word (small stages) -- bit-exact."""
+    monkeypatch.setenv("IPT_CYC_SEGSH", str(segsh))
+    for (batch, A, B, s) in [(1, 61, 47, 8), (3, 17, 19, 131), (1, 1800, 15, 480), (2, 33, 20, 12)]:
+        a = gen(batch * A * B * s, 4)
+        t = to_dev(a, 4)
+        ipt.ipt_100_(t, batch, A, B, s)
+        assert np.array_equal(to_np(t, 4), oracle.permute_inplace(a.copy(), batch, A, B, s)), (segsh, batch, A, B, s)

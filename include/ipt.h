@@ -146,6 +146,15 @@ ipt_status ipt_transpose_4stage(void *d_ptr, int64_t M, int64_t N, int64_t m, in
 ipt_status ipt_transpose_host(void *h_ptr, int64_t M, int64_t N, int elem_bytes, int queues,
                               void *d_buffer, size_t d_buffer_bytes, void *stream);
 
+/* Asynchronous form: everything is enqueued and ordered on `stream` (completion of the
+ * D2H of every panel is joined back onto `stream`); returns after enqueueing.  The host
+ * buffer and the device buffer (internal cache: one per (device, stream)) must not be
+ * reused until the stream has reached this point.  Calls on different streams overlap,
+ * e.g. the H2D of one matrix with the D2H of the previous one (both PCIe directions). */
+ipt_status ipt_transpose_host_async(void *h_ptr, int64_t M, int64_t N, int elem_bytes,
+                                    int queues, void *d_buffer, size_t d_buffer_bytes,
+                                    void *stream);
+
 /* ------------------------------------------------ elementary transpositions */
 
 /* Device workspace bytes for P(batch, A, B, s) with elem_bytes elements. */

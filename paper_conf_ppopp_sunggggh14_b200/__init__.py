@@ -69,6 +69,7 @@ ABI = [
     ("ipt_transpose_batched_plan", _int, [_vp, _i64, _i64, ctypes.POINTER(Plan), _vp, _sz, _vp]),
     ("ipt_transpose_4stage", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
     ("ipt_transpose_host", _int, [_vp, _i64, _i64, _int, _int, _vp, _sz, _vp]),
+    ("ipt_transpose_host_async", _int, [_vp, _i64, _i64, _int, _int, _vp, _sz, _vp]),
     ("ipt_stage_workspace_bytes", _sz, [_i64, _i64, _i64, _i64, _int]),
     ("ipt_100", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
     ("ipt_010", _int, [_vp, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
@@ -226,6 +227,20 @@ def transpose_host_(h, M: int, N: int, queues: int = 4, stream=None, elem_bytes:
     _check(lib().ipt_transpose_host(ctypes.c_void_p(h.data_ptr()), M, N, eb, queues, None, 0,
                                     _stream_ptr(stream)), "ipt_transpose_host")
     return h.view(N, M) if eb == h.element_size() else h
+
+
+def transpose_host_async_(h, M: int, N: int, queues: int = 4, stream=None,
+                          elem_bytes: int | None = None):
+    """Asynchronous host-delegated transpose: enqueued on `stream` (pinned `h` required);
+    synchronise the stream before reading `h`."""
+    if h.is_cuda or not h.is_contiguous():
+        raise IptError("transpose_host_async_ expects a contiguous host tensor")
+    eb = _eb(h, elem_bytes)
+    if _nelem(h, eb) != M * N:
+        raise IptError(f"elements {_nelem(h, eb)} != M*N {M * N}")
+    _check(lib().ipt_transpose_host_async(ctypes.c_void_p(h.data_ptr()), M, N, eb, queues, None, 0,
+                                          _stream_ptr(stream)), "ipt_transpose_host_async")
+    return h
 
 
 # ----------------------------------------------------------- elementary transpositions

@@ -135,18 +135,20 @@ WsCache &ws_cache() {
     return *c;
 }
 
-ipt_status get_ws(int device, void *stream, size_t need, void **out) {
+// Internal buffers are cached per (device, stream, purpose): `purpose` 0 = flag workspace,
+// 1 = host-path staging buffer.  Growing a buffer synchronises `stream` first (work
+// already enqueued on it may still use the old buffer).
+ipt_status get_ws(int device, void *stream, size_t need, void **out, int purpose = 0) {
     if (need == 0) { *out = nullptr; return IPT_OK; }
     WsCache &c = ws_cache();
     std::lock_guard<std::mutex> lk(c.mu);
-    auto key = std::make_pair(device, stream);
+    auto key = std::make_pair(device * 2 + purpose, stream);
     auto it = c.bufs.find(key);
     if (it != c.bufs.end() && it->second.second >= need) {
         *out = it->second.first;
         return IPT_OK;
     }
     if (it != c.bufs.end()) {
-        // previous work on this stream may still use the old buffer
         cudaStreamSynchronize((cudaStream_t)stream);
         cudaFree(it->second.first);
         c.bufs.erase(it);
@@ -477,11 +479,13 @@ ipt_status ipt_transpose_4stage(void *d_ptr, int64_t M, int64_t N, int64_t m, in
 // cannot be split; stages 2 and 3 work on independent instances, so the
 // N' output panels are split into Q groups, each on its own stream: stage 2 + stage 3 +
 // device-to-host copy of the group overlap with the other groups' work (Fig. 5b).
-static ipt_status host_streams(int device, int q, cudaStream_t *out) {
+static ipt_status host_streams(int device, void *caller, int q, cudaStream_t *out) {
+    // one set of Q streams per (device, caller stream): calls on different caller streams
+    // never share queues, so asynchronous host calls on two streams overlap
     static std::mutex mu;
-    static std::map<int, std::vector<cudaStream_t>> cache;
+    static std::map<std::pair<int, void *>, std::vector<cudaStream_t>> cache;
     std::lock_guard<std::mutex> lk(mu);
-    auto &v = cache[device];
+    auto &v = cache[std::make_pair(device, caller)];
     while ((int)v.size() < q) {
         cudaStream_t s;
         if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) {
@@ -496,8 +500,9 @@ static ipt_status host_streams(int device, int q, cudaStream_t *out) {
 
 static size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 
-ipt_status ipt_transpose_host(void *h_ptr, int64_t M, int64_t N, int elem_bytes, int queues,
-                              void *d_buffer, size_t d_buffer_bytes, void *stream) {
+static ipt_status transpose_host_impl(void *h_ptr, int64_t M, int64_t N, int elem_bytes,
+                                      int queues, void *d_buffer, size_t d_buffer_bytes,
+                                      void *stream, bool sync) {
     int64_t bytes = 0;
     ipt_status s = check_shape(M, N, elem_bytes, &bytes);
     if (s) return s;
@@ -532,7 +537,7 @@ ipt_status ipt_transpose_host(void *h_ptr, int64_t M, int64_t N, int elem_bytes,
     cudaStream_t st = (cudaStream_t)stream;
     if (!dbuf) {
         void *w = nullptr;
-        if ((s = get_ws(device, (void *)((uintptr_t)stream ^ 0x1), need, &w))) return s;
+        if ((s = get_ws(device, stream, need, &w, 1))) return s;
         dbuf = (char *)w;
     } else if (d_buffer_bytes < need) {
         return IPT_ERR_NO_MEMORY;
@@ -542,7 +547,7 @@ ipt_status ipt_transpose_host(void *h_ptr, int64_t M, int64_t N, int elem_bytes,
     char *cur = dws1 + align256(ws1);
     for (int g = 0; g < Q; ++g) { dwsg[g] = cur; cur += wsg[g]; }
     std::vector<cudaStream_t> qs(Q);
-    if ((s = host_streams(device, Q, qs.data()))) return s;
+    if ((s = host_streams(device, stream, Q, qs.data()))) return s;
 
     cudaError_t e = cudaMemcpyAsync(dbuf, h_ptr, (size_t)bytes, cudaMemcpyHostToDevice, st);
     if (e != cudaSuccess) return cuda_status(e);
@@ -577,10 +582,23 @@ ipt_status ipt_transpose_host(void *h_ptr, int64_t M, int64_t N, int elem_bytes,
         cudaEventRecord(done[g], qs_g);
         cudaStreamWaitEvent(st, done[g], 0);
     }
-    e = cudaStreamSynchronize(st);
-    cudaEventDestroy(ev1);
+    e = sync ? cudaStreamSynchronize(st) : cudaGetLastError();
+    cudaEventDestroy(ev1);   // released once the recorded work completes
     for (auto d : done) cudaEventDestroy(d);
     return cuda_status(e);
+}
+
+ipt_status ipt_transpose_host(void *h_ptr, int64_t M, int64_t N, int elem_bytes, int queues,
+                              void *d_buffer, size_t d_buffer_bytes, void *stream) {
+    return transpose_host_impl(h_ptr, M, N, elem_bytes, queues, d_buffer, d_buffer_bytes,
+                               stream, true);
+}
+
+ipt_status ipt_transpose_host_async(void *h_ptr, int64_t M, int64_t N, int elem_bytes,
+                                    int queues, void *d_buffer, size_t d_buffer_bytes,
+                                    void *stream) {
+    return transpose_host_impl(h_ptr, M, N, elem_bytes, queues, d_buffer, d_buffer_bytes,
+                               stream, false);
 }
 
 // ------------------------------------------- layout marshaling (Sung's DL; NEXT-3)

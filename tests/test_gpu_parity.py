@@ -507,3 +507,20 @@ def test_ipt_100_fetch_segments(monkeypatch, segsh):
         t = to_dev(a, 4)
         ipt.ipt_100_(t, batch, A, B, s)
         assert np.array_equal(to_np(t, 4), oracle.permute_inplace(a.copy(), batch, A, B, s)), (segsh, batch, A, B, s)
+
+
+def test_transpose_host_async_two_streams():
+    """Asynchronous host-delegated calls on two streams (overlapping PCIe directions)."""
+    shapes = [(1800, 7200), (720, 1800), (97, 89), (4096, 300)]
+    hs, refs = [], []
+    for (M, N) in shapes:
+        a = seeded.matrix_np(M, N, 4)
+        hs.append(torch.from_numpy(a.view(np.int32).copy()).pin_memory())
+        refs.append(oracle.transpose_inplace(a.copy(), M, N))
+    sts = [torch.cuda.Stream(), torch.cuda.Stream()]
+    for i, ((M, N), h) in enumerate(zip(shapes, hs)):
+        ipt.transpose_host_async_(h, M, N, queues=3, stream=sts[i % 2])
+    for s in sts:
+        s.synchronize()
+    for h, ref in zip(hs, refs):
+        assert np.array_equal(h.numpy().view(np.uint32), ref)

@@ -19,12 +19,15 @@ def bench(batch, A, B, s, reps=3):
     return round(2 * batch * A * B * s * 4 / (ms / 1e3) / 1e9)
 import ast
 knobs = ast.literal_eval(os.environ.get("KNOBS", "[{}]"))
+CASES = ast.literal_eval(os.environ.get("CASES", "[('S512_st1', (1, 12800, 117, 128))]"))
 for kn in knobs:
     for k in list(os.environ):
         if k.startswith("IPT_CYC"): del os.environ[k]
     os.environ.update(kn)
-    res = {"S512_st1": bench(1, 12800, 15000 // 128, 128), "S512_st3": bench(75, 100, 200, 128),
-           "S320_st3": bench(75, 160, 200, 80), "S800_st3": bench(75, 64, 200, 200), "S240_st1": bench(1, 12800, 250, 60),
-           "pow2_S512_st1": bench(1, 16384, 64, 128), "pow2_S512_st3": bench(64, 128, 128, 128),
-           "S576_st1": bench(1, 7200, 125, 144), "S640_st3": bench(125, 45, 144, 160)}
+    res = {}
+    for name, args in CASES:
+        try:
+            res[name] = bench(*args)
+        except Exception as e:
+            res[name] = str(e)[:30]
     print(json.dumps(kn), json.dumps(res), flush=True)

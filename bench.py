@@ -196,10 +196,18 @@ def main():
     from inputs import seeded
 
     assert args.warmup >= 3, "timing rules: at least 3 warm-up steps"
+    # one process per GPU; IPT_BENCH_BACKEND=gloo lets the multi-rank logic run on a
+    # single-GPU box for testing (ranks then share the device)
+    backend = os.environ.get("IPT_BENCH_BACKEND", "nccl")
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    red_dev = dev if backend == "nccl" else torch.device("cpu")
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     wl = WORKLOADS[args.workload]
     eb = wl["eb"]
     tdt = torch.int32 if eb == 4 else torch.int64
@@ -268,7 +276,7 @@ def main():
     launches = ipt.kernel_launch_count() - launches0
     clk = clocks.stop()
     elapsed_ms = t_start.elapsed_time(t_end)
-    tmax = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
+    tmax = torch.tensor([elapsed_ms], dtype=torch.float64, device=red_dev)
     if world > 1:
         dist.barrier()
         dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
@@ -395,7 +403,7 @@ def main():
         e1.record()
         torch.cuda.synchronize()
         wall = time.perf_counter() - w0
-        ems = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+        ems = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=red_dev)
         if world > 1:
             dist.all_reduce(ems, op=dist.ReduceOp.MAX)
         hb = sum(M * N * eb for (_, M, N) in hosts)

@@ -180,6 +180,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--queues", type=int, default=4)
+    ap.add_argument("--autotune", type=int, default=4,
+                    help="candidates timed by ipt_plan_autotune per shape (<2: model plan)")
     ap.add_argument("--algo", default="3stage", choices=["3stage", "4stage"],
                     help="4stage = the paper's Gustavson/Karlsson baseline (comparison only)")
     args = ap.parse_args()
@@ -229,9 +231,22 @@ def main():
             mats.append([t, M, N, 1, 0])
     torch.cuda.synchronize()
     plans = {}
-    for (_, M, N, _, _) in mats:
-        plans[(M, N)] = ipt.plan(M, N, eb, local)
-        plans[(N, M)] = ipt.plan(N, M, eb, local)
+    for (t, M, N, cnt, _) in mats:
+        if args.autotune > 1 and cnt == 1:
+            # measured plan choice (host planning, outside the timed region; data restored)
+            plans[(M, N)] = ipt.plan_autotune(t, M, N, args.autotune)
+            ipt.transpose_(t, M, N, plan_=plans[(M, N)])
+            plans[(N, M)] = ipt.plan_autotune(t, N, M, args.autotune)
+            ipt.transpose_(t, N, M, plan_=plans[(N, M)])
+        elif args.autotune > 1:
+            plans[(M, N)] = ipt.plan_autotune_batched(t, cnt, M, N, args.autotune)
+            ipt.transpose_batched_(t, cnt, M, N, plan_=plans[(M, N)])
+            plans[(N, M)] = ipt.plan_autotune_batched(t, cnt, N, M, args.autotune)
+            ipt.transpose_batched_(t, cnt, N, M, plan_=plans[(N, M)])
+        else:
+            plans[(M, N)] = ipt.plan(M, N, eb, local)
+            plans[(N, M)] = ipt.plan(N, M, eb, local)
+    torch.cuda.synchronize()
     ws_bytes = max(ipt.workspace_bytes(p, mt[3]) for mt in mats for p in (plans[(mt[1], mt[2])], plans[(mt[2], mt[1])]))
     ws = torch.empty(max(ws_bytes, 256), dtype=torch.uint8, device=dev)
     orient = [False] * len(mats)   # False: currently M x N; True: currently N x M
@@ -443,7 +458,9 @@ def main():
                        "plans": plans_cfg,
                        "l2": "no flush: every matrix exceeds the 126 MB L2" if args.workload in ("sweep", "c3", "c4", "c5") else "L2-resident (52 MB)",
                        "parallelism": f"replicas x{world}" if "batch" not in wl else f"batch shards x{world}",
-                       "algo": args.algo},
+                       "algo": args.algo,
+                       "planning": (f"ipt_plan_autotune, {args.autotune} candidates per shape "
+                                    "(before the timed region)") if args.autotune > 1 else "cost model"},
             "hbm_frac_stage_scaled": round(stage_scaled, 4) if stage_scaled else None,
             "per_shape": per_shape, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
             "clocks": clk, "verified": ok,

@@ -96,6 +96,21 @@ ipt_status ipt_plan(int64_t M, int64_t N, int elem_bytes, int device, ipt_plan_t
 ipt_status ipt_plan_with_tiles(int64_t M, int64_t N, int64_t m, int64_t n, int elem_bytes,
                                int device, ipt_plan_t *out);
 
+/* Measured plan choice: the cost model's best `candidates` plans (plus the best plan of
+ * every other stage count) each transpose the matrix at d_ptr (M x N) and the model-best
+ * N x M plan transposes it back, timed with CUDA events on `stream`; the data is
+ * unchanged on return (synchronous).  The fastest plan is returned and remembered for
+ * (M, N, elem_bytes, device): later ipt_plan / ipt_transpose calls use it.
+ * candidates < 2 returns ipt_plan's choice without timing. */
+ipt_status ipt_plan_autotune(void *d_ptr, int64_t M, int64_t N, int elem_bytes, int candidates,
+                             void *stream, ipt_plan_t *out);
+
+/* Same for a batch (timed with ipt_transpose_batched_plan on all `count` matrices); the
+ * result is returned, not remembered (single-matrix plans may differ). */
+ipt_status ipt_plan_autotune_batched(void *d_base, int64_t count, int64_t stride_bytes,
+                                     int64_t M, int64_t N, int elem_bytes, int candidates,
+                                     void *stream, ipt_plan_t *out);
+
 /* Device workspace bytes for executing `plan` on a batch of `batch` matrices. */
 size_t ipt_workspace_bytes(const ipt_plan_t *plan, int64_t batch);
 

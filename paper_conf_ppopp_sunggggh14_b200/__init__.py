@@ -61,6 +61,8 @@ _i64, _int, _vp, _sz = ctypes.c_int64, ctypes.c_int, ctypes.c_void_p, ctypes.c_s
 ABI = [
     ("ipt_plan", _int, [_i64, _i64, _int, _int, ctypes.POINTER(Plan)]),
     ("ipt_plan_with_tiles", _int, [_i64, _i64, _i64, _i64, _int, _int, ctypes.POINTER(Plan)]),
+    ("ipt_plan_autotune", _int, [_vp, _i64, _i64, _int, _int, _vp, ctypes.POINTER(Plan)]),
+    ("ipt_plan_autotune_batched", _int, [_vp, _i64, _i64, _i64, _i64, _int, _int, _vp, ctypes.POINTER(Plan)]),
     ("ipt_workspace_bytes", _sz, [ctypes.POINTER(Plan), _i64]),
     ("ipt_transpose", _int, [_vp, _i64, _i64, _int, _vp]),
     ("ipt_transpose_plan", _int, [_vp, ctypes.POINTER(Plan), _vp, _sz, _vp]),
@@ -148,6 +150,30 @@ def plan(M: int, N: int, elem_bytes: int, device: int = -1, m: int | None = None
     else:
         _check(lib().ipt_plan_with_tiles(M, N, m, n, elem_bytes, device, ctypes.byref(p)),
                "ipt_plan_with_tiles")
+    return p
+
+
+def plan_autotune(t, M: int, N: int, candidates: int = 4, stream=None,
+                  elem_bytes: int | None = None) -> Plan:
+    """Time the cost model's best candidate plans on t (data unchanged on return) and
+    remember the fastest for (M, N, elem_bytes, device)."""
+    eb = _eb(t, elem_bytes)
+    p = Plan()
+    _check(lib().ipt_plan_autotune(_dev_ptr(t), M, N, eb, candidates, _stream_ptr(stream),
+                                   ctypes.byref(p)), "ipt_plan_autotune")
+    return p
+
+
+def plan_autotune_batched(t, count: int, M: int, N: int, candidates: int = 4,
+                          stride_elems: int | None = None, stream=None,
+                          elem_bytes: int | None = None) -> Plan:
+    """plan_autotune for `count` matrices (data unchanged on return)."""
+    eb = _eb(t, elem_bytes)
+    stride = (stride_elems if stride_elems is not None else M * N) * eb
+    p = Plan()
+    _check(lib().ipt_plan_autotune_batched(_dev_ptr(t), count, stride, M, N, eb, candidates,
+                                           _stream_ptr(stream), ctypes.byref(p)),
+           "ipt_plan_autotune_batched")
     return p
 
 

@@ -20,6 +20,9 @@
 namespace ipt {
 
 ipt_status plan_search(int64_t M, int64_t N, int eb, int device, ipt_plan_t *out);
+std::vector<std::pair<int64_t, int64_t>> plan_candidates(int64_t M, int64_t N, int eb,
+                                                         int device, int k);
+void remember_tuned(int64_t M, int64_t N, int eb, int device, int64_t m, int64_t n);
 void fill_plan(int64_t M, int64_t N, int64_t m, int64_t n, int eb, int device, ipt_plan_t *out);
 
 static std::atomic<uint64_t> g_launches{0};
@@ -413,6 +416,70 @@ ipt_status ipt_1000(void *d_ptr, int64_t d0, int64_t d1, int64_t d2, int64_t d3,
     int64_t s = 0;
     if (d2 < 1 || d3 < 1 || !mul_ok(d2, d3, &s)) return IPT_ERR_INVALID_ARG;
     return ipt_100(d_ptr, 1, d0, d1, s, elem_bytes, d_workspace, ws_bytes, stream);
+}
+
+// ------------------------------------------------------------- measured plan choice
+// Sec. 7.4 says exhaustive search is too slow and prunes it; here the cost model prunes
+// to a few candidates and the device decides: each candidate transposes the caller's
+// matrix (M x N -> N x M) and the model-best N x M plan transposes it back, so the data
+// is unchanged on return.  The winner is remembered for (M, N, elem_bytes, device) and
+// returned by ipt_plan / used by ipt_transpose from then on.
+static ipt_status autotune_impl(void *d_ptr, int64_t count, int64_t stride, int64_t M,
+                                int64_t N, int elem_bytes, int candidates, void *stream,
+                                ipt_plan_t *out) {
+    if (!out || count < 1) return IPT_ERR_INVALID_ARG;
+    ipt_status s = check_shape(M, N, elem_bytes, nullptr);
+    if (s) return s;
+    if ((s = check_ptr(d_ptr, elem_bytes))) return s;
+    const int64_t mat = M * N * elem_bytes;
+    if (count == 1) stride = mat;
+    if (count > 1 && (stride < mat || stride % elem_bytes)) return IPT_ERR_INVALID_ARG;
+    const int device = current_device();
+    if (device < 0) return IPT_ERR_NO_DEVICE;
+    if (M == 1 || N == 1 || candidates < 2) return ipt_plan(M, N, elem_bytes, device, out);
+    auto cands = plan_candidates(M, N, elem_bytes, device, candidates);
+    ipt_plan_t back;
+    if ((s = plan_search(N, M, elem_bytes, device, &back))) return s;
+    cudaStream_t st = (cudaStream_t)stream;
+    cudaEvent_t e0, e1;
+    if (cudaEventCreate(&e0) != cudaSuccess || cudaEventCreate(&e1) != cudaSuccess)
+        return cuda_status(cudaGetLastError());
+    float best_ms = 0;
+    int64_t bm = cands[0].first, bn = cands[0].second;
+    for (size_t i = 0; i < cands.size(); ++i) {
+        ipt_plan_t p;
+        fill_plan(M, N, cands[i].first, cands[i].second, elem_bytes, device, &p);
+        float t_min = 0;
+        for (int rep = 0; rep < 2; ++rep) {
+            cudaEventRecord(e0, st);
+            if ((s = run_plan((char *)d_ptr, count, stride, &p, nullptr, 0, st, nullptr))) break;
+            cudaEventRecord(e1, st);
+            if ((s = run_plan((char *)d_ptr, count, stride, &back, nullptr, 0, st, nullptr))) break;
+            if (cudaEventSynchronize(e1) != cudaSuccess) { s = IPT_ERR_CUDA; break; }
+            float ms = 0;
+            cudaEventElapsedTime(&ms, e0, e1);
+            if (rep == 0 || ms < t_min) t_min = ms;
+        }
+        if (s) break;
+        if (i == 0 || t_min < best_ms) { best_ms = t_min; bm = cands[i].first; bn = cands[i].second; }
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    if (s) return s;
+    if (count == 1) remember_tuned(M, N, elem_bytes, device, bm, bn);
+    fill_plan(M, N, bm, bn, elem_bytes, device, out);
+    return IPT_OK;
+}
+
+ipt_status ipt_plan_autotune(void *d_ptr, int64_t M, int64_t N, int elem_bytes, int candidates,
+                             void *stream, ipt_plan_t *out) {
+    return autotune_impl(d_ptr, 1, 0, M, N, elem_bytes, candidates, stream, out);
+}
+
+ipt_status ipt_plan_autotune_batched(void *d_base, int64_t count, int64_t stride_bytes,
+                                     int64_t M, int64_t N, int elem_bytes, int candidates,
+                                     void *stream, ipt_plan_t *out) {
+    return autotune_impl(d_base, count, stride_bytes, M, N, elem_bytes, candidates, stream, out);
 }
 
 // ---------------------------------------------- 4-stage baseline (Fig. 2; NEXT-2)

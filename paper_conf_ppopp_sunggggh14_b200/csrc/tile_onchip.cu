@@ -190,8 +190,8 @@ __global__ void __launch_bounds__(512) tile_onchip_tma(const TileParams p) {
 }
 
 // ------------------------------------------------------------ register-staged kernel
-template <int EB, int U>
-__global__ void __launch_bounds__(512, 2) tile_onchip_ldg(const TileParams p) {
+template <int EB, int U, int MINB = 2>
+__global__ void __launch_bounds__(512, MINB) tile_onchip_ldg(const TileParams p) {
     extern __shared__ __align__(128) unsigned char smem[];
     const uint32_t sbase = smem_u32(smem);
     const uint32_t nvec = (uint32_t)(p.tile_bytes / 16);
@@ -250,8 +250,8 @@ __device__ __forceinline__ void cluster_sync_all() {
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
-template <int EB, int U>
-__global__ void __launch_bounds__(512, 2) tile_onchip_cluster(const TileParams p) {
+template <int EB, int U, int MINB = 2>
+__global__ void __launch_bounds__(512, MINB) tile_onchip_cluster(const TileParams p) {
     constexpr int V = 16 / EB;
     extern __shared__ __align__(128) unsigned char smem[];
     const uint32_t sbase = smem_u32(smem);
@@ -357,6 +357,73 @@ __device__ __forceinline__ void load_slice_vec(T *s, const T *src, uint32_t cnt,
             }
         }
     }
+}
+
+// ------------------------------------------------------------ streaming slice kernel
+// One CTA per SM (slices > 113 KB, single CTA or cluster row split): the write-out of
+// tile t and the load of tile t + 1 are overlapped inside the CTA.  The slice is processed
+// in groups of 8 V-row blocks (each group writes 8*V*elem = 128 contiguous bytes into
+// every output row); as soon as a group has been written out, the same group of the
+// next tile is fetched into the freed shared memory with cp.async (no registers, so the
+// stores of the following groups keep flowing).  The in-place rule is unchanged: no
+// store into tile t+1 before every CTA of the cluster has finished loading it.
+__device__ __forceinline__ void cp_async16(uint32_t sdst, const void *gsrc) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(sdst), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
+template <int EB>
+__global__ void __launch_bounds__(512, 1) tile_onchip_stream(const TileParams p) {
+    constexpr int V = 16 / EB;
+    constexpr uint32_t GB = 8;                       // V-row blocks per group
+    extern __shared__ __align__(128) unsigned char smem[];
+    const uint32_t sbase = smem_u32(smem);
+    const uint32_t K = p.K ? p.K : 1;
+    const uint32_t rank = (K > 1) ? cluster_rank() : 0;
+    const uint32_t cid = blockIdx.x / K, ncl = gridDim.x / K;
+    const uint32_t mv = p.m / V, nvr = p.n / V;
+    const uint32_t b0 = (uint32_t)((uint64_t)rank * mv / K);
+    const uint32_t b1 = (uint32_t)((uint64_t)(rank + 1) * mv / K);
+    const uint32_t nb = b1 - b0;
+    const uint32_t ngroups = (nb + GB - 1) / GB;
+
+    auto load_group = [&](const char *g, uint32_t grp) {   // cp.async rows of one group
+        const uint32_t bl0 = grp * GB, bl1 = min(nb, bl0 + GB);
+        const uint32_t rows = (bl1 - bl0) * V;
+        const uint32_t cnt = rows * nvr;
+        const char *src = g + ((size_t)(b0 + bl0) * V * nvr) * 16;
+        const uint32_t srow0 = bl0 * V;
+        for (uint32_t e = threadIdx.x; e < cnt; e += blockDim.x) {
+            uint32_t i, j;
+            fdivmod32(e, p.divNV32, i, j);
+            cp_async16(sbase + ((srow0 + i) * p.q + j) * 16, src + (size_t)e * 16);
+        }
+    };
+
+    uint64_t t = cid;
+    if (t < p.count) {
+        const char *g = tile_ptr(p, t);
+        for (uint32_t grp = 0; grp < ngroups; ++grp) load_group(g, grp);
+        cp_async_commit();
+    }
+    for (; t < p.count; t += ncl) {
+        char *g = tile_ptr(p, t);
+        cp_async_wait_all();
+        __syncthreads();
+        if (K > 1) cluster_sync_all();   // all slices of tile t on chip before any store
+        const uint64_t tn = t + ncl;
+        const char *gn = (tn < p.count) ? tile_ptr(p, tn) : nullptr;
+        for (uint32_t grp = 0; grp < ngroups; ++grp) {
+            const uint32_t bl0 = grp * GB, cntb = min(nb, bl0 + GB) - bl0;
+            const FastDiv32 dv = make_fastdiv32_dev(cntb);
+            write_out<EB>(p, sbase + bl0 * V * p.q * 16, g, p.q, b0 + bl0, cntb, dv, 0, nvr);
+            __syncthreads();                 // group consumed -> refill with tile t + 1
+            if (gn) load_group(gn, grp);
+            cp_async_commit();
+        }
+    }
+    cp_async_wait_all();
 }
 
 // ------------------------------------------------------------------- generic kernel
@@ -696,6 +763,15 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
         p.divMV32 = make_fastdiv32((uint32_t)(d.A / V));
         p.nbuf = tma_nbuf();
         const size_t smem = fast_smem(d.A, d.B, d.eb);
+        const bool big = smem > 113 * 1024 && env_int("IPT_TILE_BIGU", 1);
+        if (smem > 113 * 1024 && env_int("IPT_TILE_STREAM", 1) && tile_mode() != MODE_TMA) {
+            p.K = 1;
+            switch (d.eb) {
+                case 4: return go(tile_onchip_stream<4>, p, smem, st, device);
+                case 8: return go(tile_onchip_stream<8>, p, smem, st, device);
+                case 16: return go(tile_onchip_stream<16>, p, smem, st, device);
+            }
+        }
         if (tile_mode() == MODE_TMA) {
             switch (d.eb) {
                 case 4: return go(tile_onchip_tma<4>, p, smem, st, device);
@@ -704,9 +780,13 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
             }
         } else {
             switch (d.eb) {
-                case 4: return go(tile_onchip_ldg<4, 8>, p, smem, st, device);
-                case 8: return go(tile_onchip_ldg<8, 8>, p, smem, st, device);
-                case 16: return go(tile_onchip_ldg<16, 8>, p, smem, st, device);
+                // one CTA per SM for > 113 KB: twice the loads in flight per thread
+                case 4: return big ? go(tile_onchip_ldg<4, 16, 1>, p, smem, st, device)
+                                   : go(tile_onchip_ldg<4, 8>, p, smem, st, device);
+                case 8: return big ? go(tile_onchip_ldg<8, 16, 1>, p, smem, st, device)
+                                   : go(tile_onchip_ldg<8, 8>, p, smem, st, device);
+                case 16: return big ? go(tile_onchip_ldg<16, 16, 1>, p, smem, st, device)
+                                    : go(tile_onchip_ldg<16, 8>, p, smem, st, device);
             }
         }
     }
@@ -721,10 +801,22 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
             const size_t smem = p.colsplit
                 ? (size_t)d.A * (size_t)(((nvr + K - 1) / K) | 1) * 16
                 : (size_t)((d.A / V + K - 1) / K) * V * p.q * 16;
+            const bool big = smem > 113 * 1024 && env_int("IPT_TILE_BIGU", 1);
+            if (big && !p.colsplit && env_int("IPT_TILE_STREAM", 1)) {
+                p.divNV32 = make_fastdiv32((uint32_t)nvr);
+                switch (d.eb) {
+                    case 4: return go_cluster(tile_onchip_stream<4>, p, smem, K, st, device);
+                    case 8: return go_cluster(tile_onchip_stream<8>, p, smem, K, st, device);
+                    case 16: return go_cluster(tile_onchip_stream<16>, p, smem, K, st, device);
+                }
+            }
             switch (d.eb) {
-                case 4: return go_cluster(tile_onchip_cluster<4, 8>, p, smem, K, st, device);
-                case 8: return go_cluster(tile_onchip_cluster<8, 8>, p, smem, K, st, device);
-                case 16: return go_cluster(tile_onchip_cluster<16, 8>, p, smem, K, st, device);
+                case 4: return big ? go_cluster(tile_onchip_cluster<4, 16, 1>, p, smem, K, st, device)
+                                   : go_cluster(tile_onchip_cluster<4, 8>, p, smem, K, st, device);
+                case 8: return big ? go_cluster(tile_onchip_cluster<8, 16, 1>, p, smem, K, st, device)
+                                   : go_cluster(tile_onchip_cluster<8, 8>, p, smem, K, st, device);
+                case 16: return big ? go_cluster(tile_onchip_cluster<16, 16, 1>, p, smem, K, st, device)
+                                    : go_cluster(tile_onchip_cluster<16, 8>, p, smem, K, st, device);
             }
         }
     }

@@ -524,3 +524,40 @@ def test_transpose_host_async_two_streams():
         s.synchronize()
     for h, ref in zip(hs, refs):
         assert np.array_equal(h.numpy().view(np.uint32), ref)
+
+
+@pytest.mark.parametrize("eb,batch,A,B", [(4, 5, 256, 200), (8, 4, 120, 200), (16, 3, 100, 120),
+                                          (4, 3, 7200, 120), (4, 7, 1800, 160), (8, 2, 1000, 96)])
+def test_ipt_010_streaming_slices(eb, batch, A, B):
+    """One CTA per SM (slices > 113 KB): write-out of tile t overlapped with the cp.async
+    refill of tile t+1, group by group."""
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)
+
+
+def test_plan_autotune_restores_data_and_is_used():
+    M, N = 1800, 2400
+    a = seeded.matrix_np(M, N, 4)
+    t = to_dev(a, 4)
+    p = ipt.plan_autotune(t, M, N, 4)
+    assert np.array_equal(to_np(t, 4), a)               # data unchanged
+    assert M % p.m == 0 and N % p.n == 0
+    q = ipt.plan(M, N, 4, 0)                            # remembered for this device
+    assert (q.m, q.n) == (p.m, p.n)
+    ipt.transpose_(t, M, N)
+    assert np.array_equal(to_np(t, 4), oracle.transpose_inplace(a.copy(), M, N))
+
+
+def test_plan_autotune_batched_restores_data():
+    count, M, N = 6, 360, 1200
+    a = seeded.batch_np(count, M, N, 4)
+    t = to_dev(a, 4)
+    p = ipt.plan_autotune_batched(t, count, M, N, 4)
+    assert np.array_equal(to_np(t, 4), a)
+    ipt.transpose_batched_(t, count, M, N, plan_=p)
+    ref = a.copy()
+    for i in range(count):
+        oracle.transpose_inplace(ref[i * M * N:(i + 1) * M * N], M, N)
+    assert np.array_equal(to_np(t, 4), ref)

@@ -383,21 +383,31 @@ __global__ void __launch_bounds__(512, 1) tile_onchip_stream(const TileParams p)
     const uint32_t rank = (K > 1) ? cluster_rank() : 0;
     const uint32_t cid = blockIdx.x / K, ncl = gridDim.x / K;
     const uint32_t mv = p.m / V, nvr = p.n / V;
-    const uint32_t b0 = (uint32_t)((uint64_t)rank * mv / K);
-    const uint32_t b1 = (uint32_t)((uint64_t)(rank + 1) * mv / K);
-    const uint32_t nb = b1 - b0;
+    uint32_t b0, b1, c0, c1, q;
+    if (!p.colsplit) {   // row split: V-row blocks [b0, b1), all 16-byte columns
+        b0 = (uint32_t)((uint64_t)rank * mv / K);
+        b1 = (uint32_t)((uint64_t)(rank + 1) * mv / K);
+        c0 = 0; c1 = nvr; q = p.q;
+    } else {             // column split: all rows, 16-byte columns [c0, c1)
+        b0 = 0; b1 = mv;
+        c0 = (uint32_t)((uint64_t)rank * nvr / K);
+        c1 = (uint32_t)((uint64_t)(rank + 1) * nvr / K);
+        q = (c1 - c0) | 1u;
+    }
+    const uint32_t nb = b1 - b0, cvec = c1 - c0;
     const uint32_t ngroups = (nb + GB - 1) / GB;
+    const FastDiv32 divc = make_fastdiv32_dev(cvec);
 
     auto load_group = [&](const char *g, uint32_t grp) {   // cp.async rows of one group
         const uint32_t bl0 = grp * GB, bl1 = min(nb, bl0 + GB);
         const uint32_t rows = (bl1 - bl0) * V;
-        const uint32_t cnt = rows * nvr;
-        const char *src = g + ((size_t)(b0 + bl0) * V * nvr) * 16;
+        const uint32_t cnt = rows * cvec;
+        const char *src = g + ((size_t)(b0 + bl0) * V * nvr + c0) * 16;
         const uint32_t srow0 = bl0 * V;
         for (uint32_t e = threadIdx.x; e < cnt; e += blockDim.x) {
             uint32_t i, j;
-            fdivmod32(e, p.divNV32, i, j);
-            cp_async16(sbase + ((srow0 + i) * p.q + j) * 16, src + (size_t)e * 16);
+            fdivmod32(e, divc, i, j);
+            cp_async16(sbase + ((srow0 + i) * q + j) * 16, src + ((size_t)i * nvr + j) * 16);
         }
     };
 
@@ -417,7 +427,7 @@ __global__ void __launch_bounds__(512, 1) tile_onchip_stream(const TileParams p)
         for (uint32_t grp = 0; grp < ngroups; ++grp) {
             const uint32_t bl0 = grp * GB, cntb = min(nb, bl0 + GB) - bl0;
             const FastDiv32 dv = make_fastdiv32_dev(cntb);
-            write_out<EB>(p, sbase + bl0 * V * p.q * 16, g, p.q, b0 + bl0, cntb, dv, 0, nvr);
+            write_out<EB>(p, sbase + bl0 * V * q * 16, g, q, b0 + bl0, cntb, dv, c0, cvec);
             __syncthreads();                 // group consumed -> refill with tile t + 1
             if (gn) load_group(gn, grp);
             cp_async_commit();
@@ -766,6 +776,7 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
         const bool big = smem > 113 * 1024 && env_int("IPT_TILE_BIGU", 1);
         if (smem > 113 * 1024 && env_int("IPT_TILE_STREAM", 1) && tile_mode() != MODE_TMA) {
             p.K = 1;
+            p.colsplit = 0;
             switch (d.eb) {
                 case 4: return go(tile_onchip_stream<4>, p, smem, st, device);
                 case 8: return go(tile_onchip_stream<8>, p, smem, st, device);
@@ -802,7 +813,7 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
                 ? (size_t)d.A * (size_t)(((nvr + K - 1) / K) | 1) * 16
                 : (size_t)((d.A / V + K - 1) / K) * V * p.q * 16;
             const bool big = smem > 113 * 1024 && env_int("IPT_TILE_BIGU", 1);
-            if (big && !p.colsplit && env_int("IPT_TILE_STREAM", 1)) {
+            if (big && env_int("IPT_TILE_STREAM", 1)) {
                 p.divNV32 = make_fastdiv32((uint32_t)nvr);
                 switch (d.eb) {
                     case 4: return go_cluster(tile_onchip_stream<4>, p, smem, K, st, device);

@@ -283,11 +283,13 @@ def main():
     clocks = ClockSampler(local)
     launches0 = ipt.kernel_launch_count()
     orient_before = list(orient)
+    torch.cuda.nvtx.range_push("timed")       # ncu --nvtx --nvtx-include "timed/"
     t_start.record()
     for s in range(args.steps):
         one_step(evs[s] if ("batch" not in wl and args.algo == "3stage") else None)
     t_end.record()
     torch.cuda.synchronize()
+    torch.cuda.nvtx.range_pop()
     launches = ipt.kernel_launch_count() - launches0
     clk = clocks.stop()
     elapsed_ms = t_start.elapsed_time(t_end)

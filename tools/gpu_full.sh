@@ -8,7 +8,7 @@ timeout 900 python bench.py --steps 10 --warmup 3 > gpurun_out/bench.json 2> gpu
 for w in c1 c3 c4 c5; do timeout 600 python bench.py --workload $w --steps 10 --warmup 3 --no-cpu > gpurun_out/bench_$w.json 2>> gpurun_out/bench.err; done
 timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/bench_ref.json 2>> gpurun_out/bench.err
 # launch list (cold, serialised) of the default bench command: every kernel with its time and DRAM bytes
-timeout 900 $NCU --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu > gpurun_out/launches_bench.log 2>&1
+timeout 1200 $NCU --nvtx --nvtx-include "timed/" --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu > gpurun_out/launches_bench.log 2>&1
 # one full capture of each kernel kind on a sweep matrix
 timeout 900 $NCU --set full --clock-control none --import-source on -k regex:cycle_global -s 4 -c 2 -o gpurun_out/prof_cyc -f python tools/prof_one.py 12800 15000 2 > gpurun_out/prof_cyc.log 2>&1
 timeout 600 $NCU --set full --clock-control none --import-source on -k regex:tile_onchip -s 2 -c 1 -o gpurun_out/prof_tile -f python tools/prof_one.py 12800 15000 2 > gpurun_out/prof_tile.log 2>&1

@@ -48,6 +48,7 @@ struct TileParams {
     FastDiv32 divM32, divN32, divMV32, divMVK32, divNV32;   // m, n, m/V, (m/V)/K, n/V
     uint32_t K;           // cluster path: CTAs per tile
     int colsplit;         // generic cluster path: split columns (1) or rows (0)
+    uint32_t ralign;      // generic cluster row split: slice boundaries in multiples of this
     int vec16;            // generic path: tiles 16-byte aligned, 16-byte loads
 };
 
@@ -490,14 +491,24 @@ __global__ void __launch_bounds__(512, 1) tile_generic_cluster(const TileParams 
     const uint32_t rank = cluster_rank();
     const uint32_t cid = blockIdx.x / K, ncl = gridDim.x / K;
     if (!p.colsplit) {
-        // row split: CTA k holds rows [r0, r1); writes that column segment of every output row
-        const uint32_t r0 = (uint32_t)((uint64_t)rank * p.m / K);
-        const uint32_t r1 = (uint32_t)((uint64_t)(rank + 1) * p.m / K);
+        // row split: CTA k holds rows [r0, r1); writes that column segment of every output
+        // row.  Slice boundaries are rounded to RA rows so that every slice starts on a
+        // 16-byte boundary (16-byte slice loads), and -- when output rows are 16-byte
+        // multiples -- the column segments are written with 16-byte stores.
+        constexpr uint32_t PV = 16 / sizeof(T) > 0 ? 16 / sizeof(T) : 1;
+        const uint32_t ra = p.ralign ? p.ralign : 1;
+        const uint32_t units = p.m / ra;
+        const uint32_t r0 = (uint32_t)((uint64_t)rank * units / K) * ra;
+        const uint32_t r1 = (rank + 1 == K) ? p.m : (uint32_t)((uint64_t)(rank + 1) * units / K) * ra;
         const uint32_t rows = r1 - r0;
         const uint32_t cnt = rows * p.n;
         const FastDiv32 divRows = make_fastdiv32_dev(rows);
         const bool vec = p.vec16 && (((uint64_t)r0 * p.n * sizeof(T)) % 16 == 0) &&
                          (((uint64_t)cnt * sizeof(T)) % 16 == 0);
+        const bool vecst = p.vec16 && PV > 1 && ((uint64_t)p.m * sizeof(T)) % 16 == 0 &&
+                           ((uint64_t)r0 * sizeof(T)) % 16 == 0 && rows % PV == 0;
+        const uint32_t rowsv = rows / PV;
+        const FastDiv32 divRowsV = make_fastdiv32_dev(rowsv ? rowsv : 1);
         for (uint64_t t = cid; t < p.count; t += ncl) {
             T *g = reinterpret_cast<T *>(tile_ptr(p, t));
             const T *src = g + (size_t)r0 * p.n;
@@ -506,10 +517,22 @@ __global__ void __launch_bounds__(512, 1) tile_generic_cluster(const TileParams 
             else
                 load_slice_scalar<T>(s, src, cnt, p.pitch, p.divN32);
             cluster_sync_all();     // all slices loaded before any store into the tile
-            for (uint32_t o = threadIdx.x; o < cnt; o += blockDim.x) {
-                uint32_t r, cl;
-                fdivmod32(o, divRows, r, cl);   // output row r < n, column r0 + cl
-                g[(size_t)r * p.m + r0 + cl] = s[cl * p.pitch + r];
+            if (vecst) {
+                const uint32_t cntv = rowsv * p.n;
+                for (uint32_t o = threadIdx.x; o < cntv; o += blockDim.x) {
+                    uint32_t r, clv;
+                    fdivmod32(o, divRowsV, r, clv);   // output row r, columns r0 + PV*clv ..
+                    union { uint4 w; T x[PV]; } u;
+#pragma unroll
+                    for (uint32_t k = 0; k < PV; ++k) u.x[k] = s[(clv * PV + k) * p.pitch + r];
+                    stg128_na(g + (size_t)r * p.m + r0 + clv * PV, u.w);
+                }
+            } else {
+                for (uint32_t o = threadIdx.x; o < cnt; o += blockDim.x) {
+                    uint32_t r, cl;
+                    fdivmod32(o, divRows, r, cl);   // output row r < n, column r0 + cl
+                    g[(size_t)r * p.m + r0 + cl] = s[cl * p.pitch + r];
+                }
             }
             __syncthreads();
         }
@@ -717,6 +740,21 @@ static bool generic_colsplit(int64_t A, int64_t B) {
     return env_int("IPT_TILE_COLSPLIT", 0) && B > A;
 }
 
+// Row-slice alignment of the element-path cluster split: 16 / gcd(n * eb, 16) rows start
+// every slice on a 16-byte boundary (1 when that does not divide the rows evenly).
+static uint32_t generic_ralign(int64_t A, int64_t B, int eb, int K) {
+    uint32_t x = 16, g = (uint32_t)((B * eb) & 15);
+    if (g == 0) g = 16;
+    while (g) { uint32_t t = x % g; x = g; g = t; }
+    const uint32_t a = 16 / x;
+    return (A % a == 0 && A / a >= K) ? a : 1;
+}
+
+static int64_t generic_slice_rows(int64_t A, int64_t B, int eb, int K) {
+    const int64_t ra = generic_ralign(A, B, eb, K);
+    return ((A / ra + K - 1) / K) * ra;
+}
+
 int tile_generic_cluster_k(int64_t A, int64_t B, int eb, int device) {
     if (!env_int("IPT_TILE_CLUSTER", 1) || A * B >= (1ll << 31)) return 0;
     DevProps dp = dev_props(device);
@@ -729,7 +767,7 @@ int tile_generic_cluster_k(int64_t A, int64_t B, int eb, int device) {
             bytes = (size_t)A * (size_t)(((B + K - 1) / K) | 1) * eb;
         } else {
             if (A < K) break;
-            bytes = (size_t)((A + K - 1) / K) * generic_pitch(B) * eb;
+            bytes = (size_t)generic_slice_rows(A, B, eb, K) * generic_pitch(B) * eb;
         }
         if ((long)bytes <= budget) return K;
     }
@@ -842,9 +880,10 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
         if (!K) return cudaErrorInvalidValue;
         p.K = (uint32_t)K;
         p.colsplit = generic_colsplit(d.A, d.B) ? 1 : 0;
+        p.ralign = generic_ralign(d.A, d.B, d.eb, K);
         const size_t cs = p.colsplit
             ? (size_t)d.A * (size_t)(((d.B + K - 1) / K) | 1) * d.eb
-            : (size_t)((d.A + K - 1) / K) * p.pitch * d.eb;
+            : (size_t)generic_slice_rows(d.A, d.B, d.eb, K) * p.pitch * d.eb;
         switch (d.eb) {
             case 1: return go_cluster(tile_generic_cluster<uint8_t>, p, cs, K, st, device);
             case 2: return go_cluster(tile_generic_cluster<uint16_t>, p, cs, K, st, device);

@@ -75,7 +75,6 @@ struct CycParams {
     int fence;          // 1: PTX-model fences on both sides of the claim protocol
     uint32_t zero;      // 0 at run time, opaque to the compiler (address-dependency knob)
     unsigned long long *stats;  // optional diagnostics (IPT_CYC_STATS=1): round counts
-    int debug;          // diagnostics only (IPT_CYC_DEBUG), never set by the library
 };
 
 enum : int { M_FETCH = 0, M_SCAN = 1, M_START = 2, M_CHAIN = 3, M_REFRESH = 4, M_DONE = 5 };
@@ -84,7 +83,7 @@ enum : int { M_FETCH = 0, M_SCAN = 1, M_START = 2, M_CHAIN = 3, M_REFRESH = 4, M
 // trip per chain step), so it is compiled for full occupancy (8 x 256 threads = 64 warps
 // per SM, <= 32 registers) when a walker's payload is <= 16 bytes per lane.
 template <int W, int R> struct CycMinBlocks {
-    static constexpr int value = (W * R <= 16) ? 8 : ((W * R <= 32) ? 6 : 4);
+    static constexpr int value = (W * R <= 16) ? 8 : ((W * R <= 32) ? 6 : (W * R <= 64 ? 4 : 2));
 };
 
 template <int W, int G, int R, typename I>
@@ -99,7 +98,10 @@ cycle_global_kernel(const CycParams p) {
     const I A = (I)p.A, nchunk = (I)p.nchunk, nwords = (I)p.nwords;
 
     int mode = M_FETCH;
+#ifdef IPT_CYC_STATS
+    // round statistics (diagnostic build: nvcc -DIPT_CYC_STATS, tools/cyc_stats.py)
     uint32_t st_start = 0, st_abort = 0, st_step = 0, st_lost = 0, st_refresh = 0, st_iter = 0;
+#endif
     I word = 0;            // flag word (= 32 start units) being scanned
     uint32_t cw = 0;       // cached copy of that flag word
     int nb = 0;            // next bit to consider in the word
@@ -174,6 +176,7 @@ cycle_global_kernel(const CycParams p) {
             if (!pending) break;
         }
         if (!__ballot_sync(FULL, mode != M_DONE)) {
+#ifdef IPT_CYC_STATS
             if (p.stats && gl == 0) {
                 atomicAdd(p.stats + 0, (unsigned long long)st_start);
                 atomicAdd(p.stats + 1, (unsigned long long)st_abort);
@@ -182,9 +185,12 @@ cycle_global_kernel(const CycParams p) {
                 atomicAdd(p.stats + 4, (unsigned long long)st_refresh);
                 if (lane == 0) atomicAdd(p.stats + 5, (unsigned long long)st_iter);
             }
+#endif
             break;
         }
+#ifdef IPT_CYC_STATS
         ++st_iter;
+#endif
 
         // --------------------------------------------------------------- memory round
         I tgt = k;
@@ -207,13 +213,8 @@ cycle_global_kernel(const CycParams p) {
             }
         }
         uint32_t old = 0;
-        if (mode == M_CHAIN && gl == 0) {
-            if (p.debug == 1) {          // DIAGNOSTIC ONLY (wrong results): non-atomic claim
-                old = ld_relaxed_u32(fwp);
-                if (!(old & bit)) *(volatile uint32_t *)fwp = old | bit;
-            } else {
-                old = p.fence ? atom_or_acq_u32(fwp, bit) : atom_or_u32(fwp, bit);
-            }
+        if (mode == M_CHAIN && gl == 0)
+            old = p.fence ? atom_or_acq_u32(fwp, bit) : atom_or_u32(fwp, bit);
         }
         uint32_t fw = 0;
         if (mode == M_START) {
@@ -248,6 +249,7 @@ cycle_global_kernel(const CycParams p) {
             start_lost = (seen & gmask) != 0;
             fw0 = __shfl_sync(FULL, fw, g0);
         }
+#ifdef IPT_CYC_STATS
         if (p.stats) {
             st_start += (mode == M_START);
             st_abort += (mode == M_START && start_lost);
@@ -255,6 +257,7 @@ cycle_global_kernel(const CycParams p) {
             st_lost += (mode == M_CHAIN && (old & bit));
             st_refresh += (mode == M_REFRESH);
         }
+#endif
         if (mode == M_START) {
             cw |= fw0;
             if (start_lost) {
@@ -687,7 +690,6 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
     p.refresh = (int)env_int("IPT_CYC_REFRESH", 1);
     p.fence = (int)env_int("IPT_CYC_FENCE", 1);
     p.zero = 0;
-    p.debug = (int)env_int("IPT_CYC_DEBUG", 0);
     p.stats = env_int("IPT_CYC_STATS", 0) ? (unsigned long long *)ws + 8 : nullptr;
     cudaError_t e = cudaMemsetAsync(ws, 0, 256 + p.nwords * 4, st);
     if (e != cudaSuccess) return e;

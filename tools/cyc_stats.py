@@ -1,4 +1,6 @@
-"""Round statistics of cycle_global (IPT_CYC_STATS=1) for stage-like shapes."""
+"""Round statistics of cycle_global for stage-like shapes.  Needs a diagnostic build:
+    IPT_NVCC_EXTRA=-DIPT_CYC_STATS python -m paper_conf_ppopp_sunggggh14_b200.build --force
+and IPT_CYC_STATS=1 at run time."""
 import os, sys, ctypes, json
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 os.environ["IPT_CYC_STATS"] = "1"

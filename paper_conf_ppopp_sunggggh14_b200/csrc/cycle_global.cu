@@ -215,7 +215,6 @@ cycle_global_kernel(const CycParams p) {
         uint32_t old = 0;
         if (mode == M_CHAIN && gl == 0)
             old = p.fence ? atom_or_acq_u32(fwp, bit) : atom_or_u32(fwp, bit);
-        }
         uint32_t fw = 0;
         if (mode == M_START) {
             if (p.fence) {

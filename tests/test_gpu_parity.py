@@ -561,3 +561,37 @@ def test_plan_autotune_batched_restores_data():
     for i in range(count):
         oracle.transpose_inplace(ref[i * M * N:(i + 1) * M * N], M, N)
     assert np.array_equal(to_np(t, 4), ref)
+
+
+def test_idx64_path(monkeypatch):
+    """64-bit index instantiations (used when a stage has >= 2^32 units) on medium shapes."""
+    monkeypatch.setenv("IPT_CYC_IDX64", "1")
+    for (M, N) in [(1800, 720), (97, 89), (1021, 130)]:
+        for eb in (4, 8):
+            a = seeded.matrix_np(M, N, eb)
+            t = to_dev(a, eb)
+            ipt.transpose_(t, M, N)
+            assert np.array_equal(to_np(t, eb), oracle.transpose_inplace(a.copy(), M, N)), (M, N, eb)
+    a = gen(2 * 40 * 30 * 131, 4)
+    t = to_dev(a, 4)
+    ipt.ipt_100_(t, 2, 40, 30, 131)                       # realigning walker, 64-bit
+    assert np.array_equal(to_np(t, 4), oracle.permute_inplace(a.copy(), 2, 40, 30, 131))
+
+
+def test_concurrent_streams_internal_workspace():
+    """Calls on different streams use different internal workspaces and may overlap."""
+    shapes = [(1800, 2400), (2400, 1800), (720, 1000), (97, 4093)]
+    sts = [torch.cuda.Stream() for _ in shapes]
+    ts, refs = [], []
+    for (M, N) in shapes:
+        a = seeded.matrix_np(M, N, 4)
+        ts.append(to_dev(a, 4))
+        refs.append(oracle.transpose_inplace(a.copy(), M, N))
+    torch.cuda.synchronize()
+    for rep in range(3):
+        for (M, N), t, s in zip(shapes, ts, sts):
+            a, b = (M, N) if rep % 2 == 0 else (N, M)
+            ipt.transpose_(t, a, b, stream=s)
+    torch.cuda.synchronize()
+    for t, ref in zip(ts, refs):
+        assert np.array_equal(to_np(t, 4), ref)

@@ -86,8 +86,8 @@ template <int W, int R> struct CycMinBlocks {
     static constexpr int value = (W * R <= 16) ? 8 : ((W * R <= 32) ? 6 : (W * R <= 64 ? 4 : 2));
 };
 
-template <int W, int G, int R, typename I>
-__global__ void __launch_bounds__(256, CycMinBlocks<W, R>::value)
+template <int W, int G, int R, typename I, bool LA>
+__global__ void __launch_bounds__(256, CycMinBlocks<W, LA ? 2 * R : R>::value)
 cycle_global_kernel(const CycParams p) {
     using V = typename VecT<W>::type;
     constexpr unsigned FULL = 0xffffffffu;
@@ -109,11 +109,23 @@ cycle_global_kernel(const CycParams p) {
     I ubase = 0;           // unit index of (item, k = 0, chunk)
     I k = 0, k0 = 0;
     int nv = 0;            // vectors in this chunk
-    V data[R], in[R];
+    bool ahead = false;    // LA: the next target's content is already in flight (buffer b)
+    V data[R], bufa[R], bufb[R];
 #pragma unroll
-    for (int r = 0; r < R; ++r) { data[r] = V(); in[r] = V(); }
+    for (int r = 0; r < R; ++r) { data[r] = V(); bufa[r] = V(); bufb[r] = V(); }
 
-    for (;;) {
+    auto next_of = [&](I x) -> I {
+        I q, r;
+        fdivmod_t(x, p.divB.d32, p.divB.d64, q, r);
+        return r * A + q;                              // Eq. (1) on super-element offsets
+    };
+
+    // One round: work acquisition (if needed), then one memory round trip.  `in` receives
+    // (or already holds, when `ahead`) the target's content; with LA the content of the
+    // chain's following target is loaded into `nx` at the same time.  Whoever later claims
+    // that target is its only writer, so a read issued before the claim is the original
+    // value whenever the claim is won (and is discarded otherwise).
+    auto round = [&](V (&in)[R], V (&nx)[R]) -> bool {
         // ------------------------------------------------ work acquisition (no data moved)
         for (;;) {
             const unsigned need = __ballot_sync(FULL, mode == M_FETCH && gl == 0);
@@ -159,10 +171,9 @@ cycle_global_kernel(const CycParams p) {
                 const I u = word * 32 + (I)b;
                 I tk = u, ch = 0;
                 if (p.nchunk > 1) fdivmod_t(u, p.divNchunk.d32, p.divNchunk.d64, tk, ch);
-                I T, kk, q, r;
+                I T, kk;
                 fdivmod_t(tk, p.divAB.d32, p.divAB.d64, T, kk);
-                fdivmod_t(kk, p.divB.d32, p.divB.d64, q, r);
-                if (r * A + q == kk) continue;          // fixed point of Eq. (1): nothing moves
+                if (next_of(kk) == kk) continue;        // fixed point of Eq. (1): nothing moves
                 I to, ti;
                 fdivmod_t(T, p.divInner.d32, p.divInner.d64, to, ti);
                 item = p.base + (uint64_t)to * p.ostride + (uint64_t)ti * p.istride +
@@ -170,6 +181,7 @@ cycle_global_kernel(const CycParams p) {
                 ubase = T * (I)p.AB * nchunk + ch;
                 nv = (int)((ch == nchunk - 1) ? (p.nvec - (uint64_t)ch * p.cvec) : p.cvec);
                 k = k0 = kk;
+                ahead = false;
                 mode = M_START;
             }
             const unsigned pending = __ballot_sync(FULL, mode == M_FETCH || mode == M_SCAN);
@@ -186,30 +198,42 @@ cycle_global_kernel(const CycParams p) {
                 if (lane == 0) atomicAdd(p.stats + 5, (unsigned long long)st_iter);
             }
 #endif
-            break;
+            return false;
         }
 #ifdef IPT_CYC_STATS
         ++st_iter;
 #endif
 
         // --------------------------------------------------------------- memory round
-        I tgt = k;
-        if (mode == M_CHAIN) {
-            I q, r;
-            fdivmod_t(k, p.divB.d32, p.divB.d64, q, r);
-            tgt = r * A + q;                           // Eq. (1) on super-element offsets
-        }
+        const I tgt = (mode == M_CHAIN) ? next_of(k) : k;
+        // Cycle closed at our own start x: x must still be CLAIMED (another walker carrying
+        // A[prev(x)] -- the start walker of prev(x) -- may race for it), but its backup is
+        // the value this walker already delivered, so it is not re-read.
         const bool back_home = (mode == M_CHAIN) && (tgt == k0);
         const I ut = ubase + tgt * nchunk;             // flag index of the target unit
         const uint32_t bit = 1u << ((uint32_t)ut & 31);
         uint32_t *fwp = p.flags + (ut >> 5);
         char *addr = item + (uint64_t)tgt * p.S;
+        const bool moving = (mode == M_START || mode == M_CHAIN) && !back_home;
 
-        if ((mode == M_START || mode == M_CHAIN) && !back_home) {
+        if (moving && !(LA && ahead)) {
 #pragma unroll
             for (int r = 0; r < R; ++r) {
                 const int v = gl + r * G;
                 if (v < nv) in[r] = ld_cg<W>(addr + (size_t)v * W);
+            }
+        }
+        bool nx_loaded = false;
+        if (LA && moving) {
+            const I t2 = next_of(tgt);
+            if (t2 != k0) {
+                char *a2 = item + (uint64_t)t2 * p.S;
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    const int v = gl + r * G;
+                    if (v < nv) nx[r] = ld_cg<W>(a2 + (size_t)v * W);
+                }
+                nx_loaded = true;
             }
         }
         uint32_t old = 0;
@@ -265,6 +289,7 @@ cycle_global_kernel(const CycParams p) {
 #pragma unroll
                 for (int r = 0; r < R; ++r) data[r] = in[r];
                 mode = M_CHAIN;
+                ahead = nx_loaded;
             }
         } else if (mode == M_CHAIN) {
             if (!(old & bit)) {
@@ -279,6 +304,7 @@ cycle_global_kernel(const CycParams p) {
 #pragma unroll
                     for (int r = 0; r < R; ++r) data[r] = in[r];
                     k = tgt;
+                    ahead = nx_loaded;
                 }
             } else {
                 mode = p.refresh ? M_REFRESH : M_SCAN; // lost the claim: chain ends here
@@ -286,6 +312,16 @@ cycle_global_kernel(const CycParams p) {
         } else if (mode == M_REFRESH) {
             cw |= fw0;
             mode = M_SCAN;
+        }
+        return true;
+    };
+
+    // Ping-pong between the two receive buffers so that the look-ahead load of one round
+    // becomes the next round's backup without a register move (which would wait for it).
+    for (;;) {
+        if (!round(bufa, bufb)) break;
+        if (LA) {
+            if (!round(bufb, bufa)) break;
         }
     }
 }
@@ -523,9 +559,9 @@ Choice choose(const StageDesc &d) {
     return c;
 }
 
-template <int W, int G, int R, typename I>
+template <int W, int G, int R, typename I, bool LA>
 cudaError_t launch_t(const CycParams &p, cudaStream_t st, int device) {
-    auto kern = cycle_global_kernel<W, G, R, I>;
+    auto kern = cycle_global_kernel<W, G, R, I, LA>;
     static std::mutex mu;
     static std::map<int, int> occ_cache;
     int per_sm = 0;
@@ -582,15 +618,24 @@ cudaError_t launch_ua(const CycParams &p, cudaStream_t st, int device) {
 
 typedef cudaError_t (*LaunchFn)(const CycParams &, cudaStream_t, int);
 
+// The look-ahead variant (LA: the next target's load issued one round early, ping-pong
+// buffers) measured 10-25 % SLOWER on B200 at every super-element size (fewer resident
+// warps for the extra registers; DRAM already saturated by the random traffic), so it is
+// only built for experiments (-DIPT_CYC_LOOKAHEAD, IPT_CYC_LA=1).
 template <int W, int G, int R>
-LaunchFn pick_idx(bool idx32) {
-    return idx32 ? &launch_t<W, G, R, uint32_t> : &launch_t<W, G, R, uint64_t>;
+LaunchFn pick_idx(bool idx32, bool la) {
+#ifdef IPT_CYC_LOOKAHEAD
+    if (la) return idx32 ? &launch_t<W, G, R, uint32_t, true> : &launch_t<W, G, R, uint64_t, true>;
+#else
+    (void)la;
+#endif
+    return idx32 ? &launch_t<W, G, R, uint32_t, false> : &launch_t<W, G, R, uint64_t, false>;
 }
 
 #define IPT_CASE(W_, G_, R_) \
-    if (c.W == W_ && c.G == G_ && c.R == R_) return pick_idx<W_, G_, R_>(idx32);
+    if (c.W == W_ && c.G == G_ && c.R == R_) return pick_idx<W_, G_, R_>(idx32, la);
 
-LaunchFn lookup(const Choice &c, bool idx32) {
+LaunchFn lookup(const Choice &c, bool idx32, bool la) {
     if (c.ua) {
         if (c.R == 1) return idx32 ? &launch_ua<1, uint32_t> : &launch_ua<1, uint64_t>;
         if (c.R == 2) return idx32 ? &launch_ua<2, uint32_t> : &launch_ua<2, uint64_t>;
@@ -632,11 +677,12 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
     const uint64_t units = (uint64_t)d.outer * d.inner * d.A * d.B * c.nchunk;
     // 32-bit indices when every unit index (and word * 32 + 31) fits
     const bool idx32 = units + 64 < (1ull << 32) && !env_int("IPT_CYC_IDX64", 0);
-    LaunchFn fn = lookup(c, idx32);
+    const bool la = env_int("IPT_CYC_LA", 0) != 0;
+    LaunchFn fn = lookup(c, idx32, la);
     if (!fn) {  // unsupported forced shape: fall back to the widest generic walker
         c.G = 32; c.R = 4;
         if ((uint64_t)c.G * c.R < c.cvec) return cudaErrorInvalidValue;
-        fn = lookup(c, idx32);
+        fn = lookup(c, idx32, la);
         if (!fn) return cudaErrorInvalidValue;
     }
     CycParams p;

@@ -217,10 +217,13 @@ cycle_global_kernel(const CycParams p) {
         const bool moving = (mode == M_START || mode == M_CHAIN) && !back_home;
 
         if (moving && !(LA && ahead)) {
+            // a start's data loads are acquire loads: its flag re-check below is ordered
+            // after them without a full fence
+            const bool acq = (mode == M_START) && p.fence;
 #pragma unroll
             for (int r = 0; r < R; ++r) {
                 const int v = gl + r * G;
-                if (v < nv) in[r] = ld_cg<W>(addr + (size_t)v * W);
+                if (v < nv) in[r] = acq ? ld_acq<W>(addr + (size_t)v * W) : ld_cg<W>(addr + (size_t)v * W);
             }
         }
         bool nx_loaded = false;
@@ -241,9 +244,7 @@ cycle_global_kernel(const CycParams p) {
             old = p.fence ? atom_or_acq_u32(fwp, bit) : atom_or_u32(fwp, bit);
         uint32_t fw = 0;
         if (mode == M_START) {
-            if (p.fence) {
-                fence_acq_rel_gpu();
-            } else {   // address dependency on the loaded data instead of a fence
+            if (!p.fence) {   // address dependency on the loaded data instead of acquire
                 uint32_t acc = 0;
 #pragma unroll
                 for (int r = 0; r < R; ++r) {
@@ -416,10 +417,11 @@ __global__ void __launch_bounds__(256, 6) cycle_ua_kernel(const CycParams p) {
         const char *vb = (const char *)(a - (uintptr_t)(o * 4));
         const int nvv = (o + nw + 3) >> 2;              // covering 16-byte vectors
         if ((mode == M_START || mode == M_CHAIN) && !back_home) {
+            const bool acq = (mode == M_START) && p.fence;   // see cycle_global_kernel
 #pragma unroll
             for (int r = 0; r < R; ++r) {
                 const int j = lane + 32 * r;
-                if (j < nvv) in[r] = ld_cg<16>(vb + (size_t)j * 16);
+                if (j < nvv) in[r] = acq ? ld_acq<16>(vb + (size_t)j * 16) : ld_cg<16>(vb + (size_t)j * 16);
             }
         }
         uint32_t old = 0;
@@ -427,7 +429,6 @@ __global__ void __launch_bounds__(256, 6) cycle_ua_kernel(const CycParams p) {
             old = p.fence ? atom_or_acq_u32(fwp, bit) : atom_or_u32(fwp, bit);
         uint32_t fw = 0;
         if (mode == M_START) {
-            if (p.fence) fence_acq_rel_gpu();
             fw = ld_relaxed_u32(fwp);
         } else if (mode == M_REFRESH) {
             fw = ld_relaxed_u32(p.flags + word);

@@ -42,6 +42,35 @@ template <> __device__ __forceinline__ uint32_t ld_cg<1>(const void *p) {
     return v;
 }
 
+// Acquire loads (gpu scope): later memory operations of this thread are ordered after them.
+template <int W> __device__ __forceinline__ typename VecT<W>::type ld_acq(const void *p);
+template <> __device__ __forceinline__ uint4 ld_acq<16>(const void *p) {
+    uint4 v;
+    asm volatile("ld.acquire.gpu.global.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+    return v;
+}
+template <> __device__ __forceinline__ uint2 ld_acq<8>(const void *p) {
+    uint2 v;
+    asm volatile("ld.acquire.gpu.global.v2.u32 {%0,%1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p) : "memory");
+    return v;
+}
+template <> __device__ __forceinline__ uint32_t ld_acq<4>(const void *p) {
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+template <> __device__ __forceinline__ uint32_t ld_acq<2>(const void *p) {
+    uint16_t v;
+    asm volatile("ld.acquire.gpu.global.u16 %0, [%1];" : "=h"(v) : "l"(p) : "memory");
+    return v;
+}
+template <> __device__ __forceinline__ uint32_t ld_acq<1>(const void *p) {
+    uint16_t v;
+    asm volatile("ld.acquire.gpu.global.u8 %0, [%1];" : "=h"(v) : "l"(p) : "memory");
+    return v;
+}
+
 template <int W> __device__ __forceinline__ void st_cg(void *p, const typename VecT<W>::type &v);
 template <> __device__ __forceinline__ void st_cg<16>(void *p, const uint4 &v) {
     asm volatile("st.global.cg.v4.u32 [%0], {%1,%2,%3,%4};"

@@ -75,6 +75,7 @@ struct CycParams {
     int fence;          // 1: PTX-model fences on both sides of the claim protocol
     uint32_t zero;      // 0 at run time, opaque to the compiler (address-dependency knob)
     unsigned long long *stats;  // optional diagnostics (IPT_CYC_STATS=1): round counts
+    int fastloop;       // steady-state chain loop (IPT_CYC_FASTLOOP, default on)
 };
 
 enum : int { M_FETCH = 0, M_SCAN = 1, M_START = 2, M_CHAIN = 3, M_REFRESH = 4, M_DONE = 5 };
@@ -126,6 +127,54 @@ cycle_global_kernel(const CycParams p) {
     // that target is its only writer, so a read issued before the claim is the original
     // value whenever the claim is won (and is discarded otherwise).
     auto round = [&](V (&in)[R], V (&nx)[R]) -> bool {
+        // ----------------------------------------------- steady state: every walker chains
+        // Chains average ~30 steps, so most rounds of a warp are pure chain steps; this
+        // loop runs them without the acquisition / start / refresh logic (the kernel is
+        // issue-bound for small super-elements).  Same protocol as the general round.
+        if (!LA && p.fastloop && __all_sync(FULL, mode == M_CHAIN)) {
+            for (;;) {
+                const I tgt = next_of(k);
+                const bool back_home = (tgt == k0);
+                const I ut = ubase + tgt * nchunk;
+                const uint32_t bit = 1u << ((uint32_t)ut & 31);
+                char *addr = item + (uint64_t)tgt * p.S;
+                if (!back_home) {
+#pragma unroll
+                    for (int r = 0; r < R; ++r) {
+                        const int v = gl + r * G;
+                        if (v < nv) in[r] = ld_cg<W>(addr + (size_t)v * W);
+                    }
+                }
+                uint32_t old = 0;
+                if (gl == 0) {
+                    uint32_t *fwp = p.flags + (ut >> 5);
+                    old = p.fence ? atom_or_acq_u32(fwp, bit) : atom_or_u32(fwp, bit);
+                }
+                old = __shfl_sync(FULL, old, g0);
+                __syncwarp();
+                if (!(old & bit)) {
+#pragma unroll
+                    for (int r = 0; r < R; ++r) {
+                        const int v = gl + r * G;
+                        if (v < nv) st_cg<W>(addr + (size_t)v * W, data[r]);
+                    }
+                    if (back_home) {
+                        mode = M_SCAN;
+                    } else {
+#pragma unroll
+                        for (int r = 0; r < R; ++r) data[r] = in[r];
+                        k = tgt;
+                    }
+                } else {
+                    mode = p.refresh ? M_REFRESH : M_SCAN;
+                }
+#ifdef IPT_CYC_STATS
+                if (p.stats) { st_step += !(old & bit); st_lost += (old & bit) != 0; ++st_iter; }
+#endif
+                if (!__all_sync(FULL, mode == M_CHAIN)) break;
+            }
+            return true;
+        }
         // ------------------------------------------------ work acquisition (no data moved)
         for (;;) {
             const unsigned need = __ballot_sync(FULL, mode == M_FETCH && gl == 0);
@@ -736,6 +785,7 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
     p.refresh = (int)env_int("IPT_CYC_REFRESH", 1);
     p.fence = (int)env_int("IPT_CYC_FENCE", 1);
     p.zero = 0;
+    p.fastloop = (int)env_int("IPT_CYC_FASTLOOP", 1);
     p.stats = env_int("IPT_CYC_STATS", 0) ? (unsigned long long *)ws + 8 : nullptr;
     cudaError_t e = cudaMemsetAsync(ws, 0, 256 + p.nwords * 4, st);
     if (e != cudaSuccess) return e;

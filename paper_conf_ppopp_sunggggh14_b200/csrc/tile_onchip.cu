@@ -49,6 +49,7 @@ struct TileParams {
     uint32_t K;           // cluster path: CTAs per tile
     int colsplit;         // generic cluster path: split columns (1) or rows (0)
     uint32_t ralign;      // generic cluster row split: slice boundaries in multiples of this
+    uint32_t gb;          // streaming kernel: V-row blocks per group (0 = automatic)
     int vec16;            // generic path: tiles 16-byte aligned, 16-byte loads
 };
 
@@ -377,7 +378,6 @@ __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wai
 template <int EB>
 __global__ void __launch_bounds__(512, 1) tile_onchip_stream(const TileParams p) {
     constexpr int V = 16 / EB;
-    constexpr uint32_t GB = 8;                       // V-row blocks per group
     extern __shared__ __align__(128) unsigned char smem[];
     const uint32_t sbase = smem_u32(smem);
     const uint32_t K = p.K ? p.K : 1;
@@ -396,6 +396,9 @@ __global__ void __launch_bounds__(512, 1) tile_onchip_stream(const TileParams p)
         q = (c1 - c0) | 1u;
     }
     const uint32_t nb = b1 - b0, cvec = c1 - c0;
+    // V-row blocks per group (measured, tools/tile_sweep.py with IPT_TILE_GROUP): 8 for
+    // column slices, 16 for row slices (32 when rows are narrow)
+    const uint32_t GB = p.gb ? p.gb : (p.colsplit ? 8u : (cvec >= 24 ? 16u : 32u));
     const uint32_t ngroups = (nb + GB - 1) / GB;
     const FastDiv32 divc = make_fastdiv32_dev(cvec);
 
@@ -800,6 +803,7 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
     p.n = (uint32_t)d.B;
     p.divM = make_fastdiv((uint64_t)d.A);
     p.divN = make_fastdiv((uint64_t)d.B);
+    p.gb = (uint32_t)env_int("IPT_TILE_GROUP", 0);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) <= budget) {
         const int V = 16 / d.eb;

@@ -1,4 +1,3 @@
 cd $GRAFT_REPO_ROOT
-timeout 600 python -m pytest tests/test_gpu_parity.py -q -x --timeout 300 -p no:cacheprovider -k "010" > gpurun_out/pytest_gpu.log 2>&1; echo "rc=$?" >> gpurun_out/pytest_gpu.log
-export SHAPES="[(8192,113),(9998,64),(14803,32),(64,9998),(4999,32),(8192,131)]"
-timeout 300 python tools/tile_sweep.py > gpurun_out/tile_sweep.log 2>&1
+export SHAPES="[(7200,120),(10000,64),(120,7200),(256,200)]"
+for g in 0 8 16 32 0; do IPT_TILE_GROUP=$g timeout 300 python tools/tile_sweep.py | sed "s/^/GB=$g /" >> gpurun_out/tile_sweep.log 2>&1; done

@@ -87,8 +87,8 @@ template <int W, int R> struct CycMinBlocks {
     static constexpr int value = (W * R <= 16) ? 8 : ((W * R <= 32) ? 6 : (W * R <= 64 ? 4 : 2));
 };
 
-template <int W, int G, int R, typename I, bool LA>
-__global__ void __launch_bounds__(256, CycMinBlocks<W, LA ? 2 * R : R>::value)
+template <int W, int G, int R, typename I>
+__global__ void __launch_bounds__(256, CycMinBlocks<W, R>::value)
 cycle_global_kernel(const CycParams p) {
     using V = typename VecT<W>::type;
     constexpr unsigned FULL = 0xffffffffu;
@@ -110,10 +110,9 @@ cycle_global_kernel(const CycParams p) {
     I ubase = 0;           // unit index of (item, k = 0, chunk)
     I k = 0, k0 = 0;
     int nv = 0;            // vectors in this chunk
-    bool ahead = false;    // LA: the next target's content is already in flight (buffer b)
-    V data[R], bufa[R], bufb[R];
+    V data[R], in[R];
 #pragma unroll
-    for (int r = 0; r < R; ++r) { data[r] = V(); bufa[r] = V(); bufb[r] = V(); }
+    for (int r = 0; r < R; ++r) { data[r] = V(); in[r] = V(); }
 
     auto next_of = [&](I x) -> I {
         I q, r;
@@ -121,17 +120,16 @@ cycle_global_kernel(const CycParams p) {
         return r * A + q;                              // Eq. (1) on super-element offsets
     };
 
-    // One round: work acquisition (if needed), then one memory round trip.  `in` receives
-    // (or already holds, when `ahead`) the target's content; with LA the content of the
-    // chain's following target is loaded into `nx` at the same time.  Whoever later claims
-    // that target is its only writer, so a read issued before the claim is the original
-    // value whenever the claim is won (and is discarded otherwise).
-    auto round = [&](V (&in)[R], V (&nx)[R]) -> bool {
+    // One round: work acquisition (if needed), then one memory round trip; `in` receives
+    // the target's content.  (A variant that also loaded the chain's following target one
+    // round early -- valid, since a won claim means nobody else ever wrote it -- measured
+    // 10-25 % slower on B200: more registers, fewer warps, DRAM already saturated.)
+    auto round = [&]() -> bool {
         // ----------------------------------------------- steady state: every walker chains
         // Chains average ~30 steps, so most rounds of a warp are pure chain steps; this
         // loop runs them without the acquisition / start / refresh logic (the kernel is
         // issue-bound for small super-elements).  Same protocol as the general round.
-        if (!LA && p.fastloop && __all_sync(FULL, mode == M_CHAIN)) {
+        if (p.fastloop && __all_sync(FULL, mode == M_CHAIN)) {
             for (;;) {
                 const I tgt = next_of(k);
                 const bool back_home = (tgt == k0);
@@ -230,7 +228,6 @@ cycle_global_kernel(const CycParams p) {
                 ubase = T * (I)p.AB * nchunk + ch;
                 nv = (int)((ch == nchunk - 1) ? (p.nvec - (uint64_t)ch * p.cvec) : p.cvec);
                 k = k0 = kk;
-                ahead = false;
                 mode = M_START;
             }
             const unsigned pending = __ballot_sync(FULL, mode == M_FETCH || mode == M_SCAN);
@@ -265,7 +262,7 @@ cycle_global_kernel(const CycParams p) {
         char *addr = item + (uint64_t)tgt * p.S;
         const bool moving = (mode == M_START || mode == M_CHAIN) && !back_home;
 
-        if (moving && !(LA && ahead)) {
+        if (moving) {
             // a start's data loads are acquire loads: its flag re-check below is ordered
             // after them without a full fence
             const bool acq = (mode == M_START) && p.fence;
@@ -273,19 +270,6 @@ cycle_global_kernel(const CycParams p) {
             for (int r = 0; r < R; ++r) {
                 const int v = gl + r * G;
                 if (v < nv) in[r] = acq ? ld_acq<W>(addr + (size_t)v * W) : ld_cg<W>(addr + (size_t)v * W);
-            }
-        }
-        bool nx_loaded = false;
-        if (LA && moving) {
-            const I t2 = next_of(tgt);
-            if (t2 != k0) {
-                char *a2 = item + (uint64_t)t2 * p.S;
-#pragma unroll
-                for (int r = 0; r < R; ++r) {
-                    const int v = gl + r * G;
-                    if (v < nv) nx[r] = ld_cg<W>(a2 + (size_t)v * W);
-                }
-                nx_loaded = true;
             }
         }
         uint32_t old = 0;
@@ -339,7 +323,6 @@ cycle_global_kernel(const CycParams p) {
 #pragma unroll
                 for (int r = 0; r < R; ++r) data[r] = in[r];
                 mode = M_CHAIN;
-                ahead = nx_loaded;
             }
         } else if (mode == M_CHAIN) {
             if (!(old & bit)) {
@@ -354,7 +337,6 @@ cycle_global_kernel(const CycParams p) {
 #pragma unroll
                     for (int r = 0; r < R; ++r) data[r] = in[r];
                     k = tgt;
-                    ahead = nx_loaded;
                 }
             } else {
                 mode = p.refresh ? M_REFRESH : M_SCAN; // lost the claim: chain ends here
@@ -366,13 +348,7 @@ cycle_global_kernel(const CycParams p) {
         return true;
     };
 
-    // Ping-pong between the two receive buffers so that the look-ahead load of one round
-    // becomes the next round's backup without a register move (which would wait for it).
-    for (;;) {
-        if (!round(bufa, bufb)) break;
-        if (LA) {
-            if (!round(bufb, bufa)) break;
-        }
+    while (round()) {
     }
 }
 
@@ -609,9 +585,9 @@ Choice choose(const StageDesc &d) {
     return c;
 }
 
-template <int W, int G, int R, typename I, bool LA>
+template <int W, int G, int R, typename I>
 cudaError_t launch_t(const CycParams &p, cudaStream_t st, int device) {
-    auto kern = cycle_global_kernel<W, G, R, I, LA>;
+    auto kern = cycle_global_kernel<W, G, R, I>;
     static std::mutex mu;
     static std::map<int, int> occ_cache;
     int per_sm = 0;
@@ -668,24 +644,15 @@ cudaError_t launch_ua(const CycParams &p, cudaStream_t st, int device) {
 
 typedef cudaError_t (*LaunchFn)(const CycParams &, cudaStream_t, int);
 
-// The look-ahead variant (LA: the next target's load issued one round early, ping-pong
-// buffers) measured 10-25 % SLOWER on B200 at every super-element size (fewer resident
-// warps for the extra registers; DRAM already saturated by the random traffic), so it is
-// only built for experiments (-DIPT_CYC_LOOKAHEAD, IPT_CYC_LA=1).
 template <int W, int G, int R>
-LaunchFn pick_idx(bool idx32, bool la) {
-#ifdef IPT_CYC_LOOKAHEAD
-    if (la) return idx32 ? &launch_t<W, G, R, uint32_t, true> : &launch_t<W, G, R, uint64_t, true>;
-#else
-    (void)la;
-#endif
-    return idx32 ? &launch_t<W, G, R, uint32_t, false> : &launch_t<W, G, R, uint64_t, false>;
+LaunchFn pick_idx(bool idx32) {
+    return idx32 ? &launch_t<W, G, R, uint32_t> : &launch_t<W, G, R, uint64_t>;
 }
 
 #define IPT_CASE(W_, G_, R_) \
-    if (c.W == W_ && c.G == G_ && c.R == R_) return pick_idx<W_, G_, R_>(idx32, la);
+    if (c.W == W_ && c.G == G_ && c.R == R_) return pick_idx<W_, G_, R_>(idx32);
 
-LaunchFn lookup(const Choice &c, bool idx32, bool la) {
+LaunchFn lookup(const Choice &c, bool idx32) {
     if (c.ua) {
         if (c.R == 1) return idx32 ? &launch_ua<1, uint32_t> : &launch_ua<1, uint64_t>;
         if (c.R == 2) return idx32 ? &launch_ua<2, uint32_t> : &launch_ua<2, uint64_t>;
@@ -727,12 +694,11 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
     const uint64_t units = (uint64_t)d.outer * d.inner * d.A * d.B * c.nchunk;
     // 32-bit indices when every unit index (and word * 32 + 31) fits
     const bool idx32 = units + 64 < (1ull << 32) && !env_int("IPT_CYC_IDX64", 0);
-    const bool la = env_int("IPT_CYC_LA", 0) != 0;
-    LaunchFn fn = lookup(c, idx32, la);
+    LaunchFn fn = lookup(c, idx32);
     if (!fn) {  // unsupported forced shape: fall back to the widest generic walker
         c.G = 32; c.R = 4;
         if ((uint64_t)c.G * c.R < c.cvec) return cudaErrorInvalidValue;
-        fn = lookup(c, idx32, la);
+        fn = lookup(c, idx32);
         if (!fn) return cudaErrorInvalidValue;
     }
     CycParams p;

@@ -256,7 +256,8 @@ def main():
             a, b = (N, M) if orient[i] else (M, N)
             p = plans[(a, b)]
             if cnt > 1:
-                ipt.transpose_batched_(t, cnt, a, b, plan_=p)
+                ipt.transpose_batched_(t, cnt, a, b, plan_=p,
+                                       events=evs[i] if evs is not None else None)
             elif args.algo == "4stage":      # the paper's 4-stage baseline
                 ipt.transpose_4stage_(t, a, b, p.m, p.n)
             else:
@@ -286,7 +287,7 @@ def main():
     torch.cuda.nvtx.range_push("timed")       # ncu --nvtx --nvtx-include "timed/"
     t_start.record()
     for s in range(args.steps):
-        one_step(evs[s] if ("batch" not in wl and args.algo == "3stage") else None)
+        one_step(evs[s] if args.algo == "3stage" else None)
     t_end.record()
     torch.cuda.synchronize()
     torch.cuda.nvtx.range_pop()
@@ -314,7 +315,7 @@ def main():
     kern_n = {"cycle_global": 0, "tile_onchip": 0}
     stage_scaled = None
     per_shape = {}
-    if "batch" not in wl and args.algo == "3stage":
+    if args.algo == "3stage":
         orient_sim = list(orient_before)
         S_bytes = 0
         for s in range(args.steps):
@@ -328,17 +329,18 @@ def main():
                         continue
                     dt = evs[s][i][st].elapsed_time(evs[s][i][st + 1])
                     kern_t[v] += dt
-                    kern_bytes[v] += 2 * a * b * eb
+                    kern_bytes[v] += 2 * a * b * eb * cnt
                     kern_n[v] += 1
-                    S_bytes += 2 * a * b * eb
+                    S_bytes += 2 * a * b * eb * cnt
                     ps["ms"] += dt
                     ps["stage_ms"][st] += dt
                 ps["n"] += 1
                 orient_sim[i] = not orient_sim[i]
         for key, ps in per_shape.items():
             a, b = (int(x) for x in key.split("x"))
-            ps["eff_gbs"] = round(2 * a * b * eb * ps["n"] / (ps["ms"] / 1e3) / 1e9, 1)
-            ps["stage_gbs"] = [round(2 * a * b * eb * ps["n"] / (x / 1e3) / 1e9, 1) if x else None
+            cnt = mats[0][3] if "batch" in wl else 1
+            ps["eff_gbs"] = round(2 * a * b * eb * cnt * ps["n"] / (ps["ms"] / 1e3) / 1e9, 1)
+            ps["stage_gbs"] = [round(2 * a * b * eb * cnt * ps["n"] / (x / 1e3) / 1e9, 1) if x else None
                                for x in ps["stage_ms"]]
             del ps["ms"], ps["stage_ms"]
         stage_scaled = (S_bytes / (elapsed_ms / 1e3) / 1e9) / peak

@@ -140,6 +140,13 @@ ipt_status ipt_transpose_batched_plan(void *d_base, int64_t count, int64_t strid
                                       const ipt_plan_t *plan, void *d_workspace,
                                       size_t ws_bytes, void *stream);
 
+/* As ipt_transpose_batched_plan, recording `events` (cudaEvent_t[4], each may be NULL)
+ * around the stages as ipt_transpose_plan_events does. */
+ipt_status ipt_transpose_batched_plan_events(void *d_base, int64_t count, int64_t stride_bytes,
+                                             const ipt_plan_t *plan, void *d_workspace,
+                                             size_t ws_bytes, void *stream,
+                                             void *const *events);
+
 /* The paper's 4-stage Gustavson/Karlsson baseline (Fig. 2): 0100!, 0010!, 1000!,
  * 0100! on the 4-D view M' x m x N' x n, with the same kernels.  m | M, n | N, or 0 to
  * take the 3-stage planner's tiles.  Kept to reproduce the paper's 3-stage vs 4-stage
@@ -172,7 +179,8 @@ ipt_status ipt_transpose_host_async(void *h_ptr, int64_t M, int64_t N, int elem_
 
 /* ------------------------------------------------ elementary transpositions */
 
-/* Device workspace bytes for P(batch, A, B, s) with elem_bytes elements. */
+/* Device workspace bytes for P(batch, A, B, s) with elem_bytes elements (for s == 1 it
+ * also covers the on-chip tile kernels' group counters, 8 KB). */
 size_t ipt_stage_workspace_bytes(int64_t batch, int64_t A, int64_t B, int64_t s,
                                  int elem_bytes);
 
@@ -182,7 +190,9 @@ ipt_status ipt_100(void *d_ptr, int64_t batch, int64_t A, int64_t B, int64_t s,
                    int elem_bytes, void *d_workspace, size_t ws_bytes, void *stream);
 
 /* 010! (AoS -> ASTA, Sec. 5.1): batch x [A x B] -> batch x [B x A] (tile-local
- * transposes; on-chip when a tile fits shared memory, else cycle following). */
+ * transposes; on-chip when a tile fits the shared memory of one CTA, a cluster or a
+ * co-resident group of CTAs (up to ~16 MB of 16-byte-vectorisable tiles), else cycle
+ * following).  A given workspace must hold ipt_stage_workspace_bytes(batch, A, B, 1). */
 ipt_status ipt_010(void *d_ptr, int64_t batch, int64_t A, int64_t B, int elem_bytes,
                    void *d_workspace, size_t ws_bytes, void *stream);
 

@@ -69,6 +69,8 @@ ABI = [
     ("ipt_transpose_plan_events", _int, [_vp, ctypes.POINTER(Plan), _vp, _sz, _vp, ctypes.POINTER(_vp)]),
     ("ipt_transpose_batched", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp]),
     ("ipt_transpose_batched_plan", _int, [_vp, _i64, _i64, ctypes.POINTER(Plan), _vp, _sz, _vp]),
+    ("ipt_transpose_batched_plan_events", _int,
+     [_vp, _i64, _i64, ctypes.POINTER(Plan), _vp, _sz, _vp, ctypes.POINTER(_vp)]),
     ("ipt_transpose_4stage", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
     ("ipt_transpose_host", _int, [_vp, _i64, _i64, _int, _int, _vp, _sz, _vp]),
     ("ipt_transpose_host_async", _int, [_vp, _i64, _i64, _int, _int, _vp, _sz, _vp]),
@@ -214,14 +216,22 @@ def transpose_(t, M: int, N: int, plan_: Plan | None = None, workspace=None, str
 
 
 def transpose_batched_(t, count: int, M: int, N: int, stride_elems: int | None = None,
-                       plan_: Plan | None = None, stream=None, elem_bytes: int | None = None):
-    """count matrices of M x N at t + i*stride (elements) -> their transposes in place."""
+                       plan_: Plan | None = None, stream=None, elem_bytes: int | None = None,
+                       events=None):
+    """count matrices of M x N at t + i*stride (elements) -> their transposes in place.
+    `events` (4 torch.cuda.Event or None) are recorded around the stages (needs plan_)."""
     eb = _eb(t, elem_bytes)
     stride = (stride_elems if stride_elems is not None else M * N) * eb
     if count and (count - 1) * (stride // eb) + M * N > _nelem(t, eb):
         raise IptError("tensor too small for the batch")
     ptr, st = _dev_ptr(t), _stream_ptr(stream)
-    if plan_ is None:
+    if events is not None:
+        if plan_ is None:
+            raise IptError("events need an explicit plan")
+        _check(lib().ipt_transpose_batched_plan_events(ptr, count, stride, ctypes.byref(plan_),
+                                                       None, 0, st, _events_arr(events)),
+               "ipt_transpose_batched_plan_events")
+    elif plan_ is None:
         _check(lib().ipt_transpose_batched(ptr, count, stride, M, N, eb, st),
                "ipt_transpose_batched")
     else:

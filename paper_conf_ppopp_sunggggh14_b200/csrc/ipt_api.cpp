@@ -211,8 +211,10 @@ size_t batched_ws(const ipt_plan_t *p, int64_t count) {
     StageDesc st[3];
     plan_stages(p, nullptr, count, p->M * p->N * p->elem_bytes, st);
     size_t ws = 0;
-    for (int i = 0; i < 3; ++i)
+    for (int i = 0; i < 3; ++i) {
         if (p->variant[i] == IPT_VAR_CYCLE_GLOBAL) ws = std::max(ws, cycle_ws_bytes(st[i]));
+        if (p->variant[i] == IPT_VAR_TILE_ONCHIP) ws = std::max(ws, kTileWsBytes);
+    }
     return ws;
 }
 
@@ -234,7 +236,7 @@ ipt_status run_plan(char *base, int64_t count, int64_t stride, const ipt_plan_t 
         cudaError_t e = cudaSuccess;
         switch (p->variant[i]) {
             case IPT_VAR_IDENTITY: break;
-            case IPT_VAR_TILE_ONCHIP: e = launch_tile_onchip(sd[i], st, device); break;
+            case IPT_VAR_TILE_ONCHIP: e = launch_tile_onchip(sd[i], ws, st, device); break;
             case IPT_VAR_CYCLE_ONCHIP:   // not built yet: global-flag cycle following
             case IPT_VAR_CYCLE_GLOBAL: e = launch_cycle_global(sd[i], ws, st, device); break;
         }
@@ -303,9 +305,10 @@ ipt_status ipt_transpose(void *d_ptr, int64_t M, int64_t N, int elem_bytes, void
                     nullptr);
 }
 
-ipt_status ipt_transpose_batched_plan(void *d_base, int64_t count, int64_t stride_bytes,
-                                      const ipt_plan_t *plan, void *d_workspace,
-                                      size_t ws_bytes, void *stream) {
+ipt_status ipt_transpose_batched_plan_events(void *d_base, int64_t count, int64_t stride_bytes,
+                                             const ipt_plan_t *plan, void *d_workspace,
+                                             size_t ws_bytes, void *stream,
+                                             void *const *events) {
     ipt_status s = validate_plan(plan);
     if (s) return s;
     if (count < 0) return IPT_ERR_INVALID_ARG;
@@ -317,7 +320,14 @@ ipt_status ipt_transpose_batched_plan(void *d_base, int64_t count, int64_t strid
     int64_t tot = 0;
     if (!mul_ok(count - 1, stride_bytes, &tot) || tot > INT64_MAX - mat) return IPT_ERR_INVALID_ARG;
     return run_plan((char *)d_base, count, stride_bytes, plan, d_workspace, ws_bytes,
-                    (cudaStream_t)stream, nullptr);
+                    (cudaStream_t)stream, events);
+}
+
+ipt_status ipt_transpose_batched_plan(void *d_base, int64_t count, int64_t stride_bytes,
+                                      const ipt_plan_t *plan, void *d_workspace,
+                                      size_t ws_bytes, void *stream) {
+    return ipt_transpose_batched_plan_events(d_base, count, stride_bytes, plan, d_workspace,
+                                             ws_bytes, stream, nullptr);
 }
 
 ipt_status ipt_transpose_batched(void *d_base, int64_t count, int64_t stride_bytes, int64_t M,
@@ -360,7 +370,8 @@ static StageDesc stage_desc(void *d, int64_t batch, int64_t A, int64_t B, int64_
 size_t ipt_stage_workspace_bytes(int64_t batch, int64_t A, int64_t B, int64_t s, int elem_bytes) {
     if (check_stage((void *)16, batch, A, B, s, elem_bytes) != IPT_OK) return 0;
     if (batch == 0 || A == 1 || B == 1) return 0;
-    return cycle_ws_bytes(stage_desc(nullptr, batch, A, B, s, elem_bytes));
+    const size_t c = cycle_ws_bytes(stage_desc(nullptr, batch, A, B, s, elem_bytes));
+    return s == 1 ? std::max(c, kTileWsBytes) : c;
 }
 
 static ipt_status run_cycle(void *d, int64_t batch, int64_t A, int64_t B, int64_t s, int eb,
@@ -394,7 +405,13 @@ ipt_status ipt_010(void *d_ptr, int64_t batch, int64_t A, int64_t B, int elem_by
     if (device < 0) return IPT_ERR_NO_DEVICE;
     if (tile_onchip_fits(A, B, elem_bytes, device)) {
         StageDesc sd = stage_desc(d_ptr, batch, A, B, 1, elem_bytes);
-        return cuda_status(launch_tile_onchip(sd, (cudaStream_t)stream, device));
+        void *ws = d_workspace;
+        if (!ws) {
+            if ((st = get_ws(device, stream, kTileWsBytes, &ws))) return st;
+        } else if (ws_bytes < kTileWsBytes) {
+            return IPT_ERR_NO_MEMORY;
+        }
+        return cuda_status(launch_tile_onchip(sd, ws, (cudaStream_t)stream, device));
     }
     return run_cycle(d_ptr, batch, A, B, 1, elem_bytes, d_workspace, ws_bytes, stream);
 }
@@ -522,7 +539,11 @@ ipt_status ipt_transpose_4stage(void *d_ptr, int64_t M, int64_t N, int64_t m, in
     for (int i = 0; i < 4; ++i) {
         sd[i].ostride = sd[i].A * sd[i].B * sd[i].s * elem_bytes;
         if (sd[i].A == 1 || sd[i].B == 1) continue;
-        if (i == 1 && tile_onchip_fits(m, n, elem_bytes, device)) { tile2 = true; continue; }
+        if (i == 1 && tile_onchip_fits(m, n, elem_bytes, device)) {
+            tile2 = true;
+            need = std::max(need, kTileWsBytes);
+            continue;
+        }
         need = std::max(need, cycle_ws_bytes(sd[i]));
     }
     void *ws = d_workspace;
@@ -533,7 +554,7 @@ ipt_status ipt_transpose_4stage(void *d_ptr, int64_t M, int64_t N, int64_t m, in
     }
     for (int i = 0; i < 4; ++i) {
         if (sd[i].A == 1 || sd[i].B == 1) continue;
-        cudaError_t e = (i == 1 && tile2) ? launch_tile_onchip(sd[i], (cudaStream_t)stream, device)
+        cudaError_t e = (i == 1 && tile2) ? launch_tile_onchip(sd[i], ws, (cudaStream_t)stream, device)
                                           : launch_cycle_global(sd[i], ws, (cudaStream_t)stream, device);
         if (e != cudaSuccess) return cuda_status(e);
     }
@@ -595,6 +616,7 @@ static ipt_status transpose_host_impl(void *h_ptr, int64_t M, int64_t N, int ele
         b.inner = g0[g + 1] - g0[g];
         size_t w = 0;
         if (p.variant[1] == IPT_VAR_CYCLE_GLOBAL) w = std::max(w, cycle_ws_bytes(a));
+        if (p.variant[1] == IPT_VAR_TILE_ONCHIP) w = std::max(w, kTileWsBytes);
         if (p.variant[2] == IPT_VAR_CYCLE_GLOBAL) w = std::max(w, cycle_ws_bytes(b));
         wsg[g] = align256(w);
     }
@@ -637,7 +659,7 @@ static ipt_status transpose_host_impl(void *h_ptr, int64_t M, int64_t N, int ele
         StageDesc a = sd[1], b = sd[2];
         a.base = gb; a.inner = np_g * p.Mp;
         b.base = gb; b.inner = np_g;
-        if (p.variant[1] == IPT_VAR_TILE_ONCHIP) e = launch_tile_onchip(a, qs_g, device);
+        if (p.variant[1] == IPT_VAR_TILE_ONCHIP) e = launch_tile_onchip(a, dwsg[g], qs_g, device);
         else if (p.variant[1] == IPT_VAR_CYCLE_GLOBAL) e = launch_cycle_global(a, dwsg[g], qs_g, device);
         if (e != cudaSuccess) return cuda_status(e);
         if (p.variant[2] == IPT_VAR_CYCLE_GLOBAL) e = launch_cycle_global(b, dwsg[g], qs_g, device);

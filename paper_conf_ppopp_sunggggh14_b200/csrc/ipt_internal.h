@@ -88,11 +88,19 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
 bool tile_onchip_fits(int64_t A, int64_t B, int eb, int device);
 // 0: does not fit, 1: generic element path, 2: 16-byte path in one CTA,
 // 3: 16-byte path split over a thread-block cluster (tile_cluster_k CTAs),
-// 4: element path split over a thread-block cluster
+// 4: element path split over a thread-block cluster,
+// 5: 16-byte path split over a co-resident group of CTAs (double-buffered slices)
 int tile_onchip_path(int64_t A, int64_t B, int eb, int device);
 int tile_cluster_k(int64_t A, int64_t B, int eb, int device);
 int tile_generic_cluster_k(int64_t A, int64_t B, int eb, int device);
-cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device);
+bool tile_group_split(int64_t A, int64_t B, int eb, int device);
+// Group split of `count` tiles: CTAs per tile (0 = does not fit) and groups in flight.
+int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups);
+// Workspace of a tile stage: the group split's arrival counters (one per group,
+// kGroupCtrStride bytes apart, at most 256 groups).  `ws` may be NULL for the other paths.
+constexpr uint32_t kGroupCtrStride = 32;
+constexpr size_t kTileWsBytes = 256 * kGroupCtrStride;
+cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, int device);
 
 // Device properties used by planner and launchers (cached).
 struct DevProps {

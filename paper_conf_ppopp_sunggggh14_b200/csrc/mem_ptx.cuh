@@ -177,9 +177,26 @@ __device__ __forceinline__ uint4 lds128(uint32_t saddr) {
                  : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(saddr) : "memory");
     return v;
 }
+#ifndef IPT_ST_HINT
+#define IPT_ST_HINT 0
+#endif
 __device__ __forceinline__ void stg128_na(void *p, const uint4 &v) {
+#if IPT_ST_HINT == 1
+    asm volatile("st.global.cs.v4.u32 [%0], {%1,%2,%3,%4};"
+                 :: "l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+#elif IPT_ST_HINT == 2 || IPT_ST_HINT == 3
+    asm volatile("{\n\t.reg .b64 pol;\n\t"
+#if IPT_ST_HINT == 2
+                 "createpolicy.fractional.L2::evict_first.b64 pol, 1.0;\n\t"
+#else
+                 "createpolicy.fractional.L2::evict_last.b64 pol, 1.0;\n\t"
+#endif
+                 "st.global.L1::no_allocate.L2::cache_hint.v4.u32 [%0], {%1,%2,%3,%4}, pol;\n\t}"
+                 :: "l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+#else
     asm volatile("st.global.L1::no_allocate.v4.u32 [%0], {%1,%2,%3,%4};"
                  :: "l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+#endif
 }
 
 }  // namespace ipt

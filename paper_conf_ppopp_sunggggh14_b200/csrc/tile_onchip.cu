@@ -50,6 +50,7 @@ struct TileParams {
     int colsplit;         // generic cluster path: split columns (1) or rows (0)
     uint32_t ralign;      // generic cluster row split: slice boundaries in multiples of this
     uint32_t gb;          // streaming kernel: V-row blocks per group (0 = automatic)
+    uint32_t *gbar;       // group-split kernel: one arrival counter per group (workspace)
     int vec16;            // generic path: tiles 16-byte aligned, 16-byte loads
 };
 
@@ -440,6 +441,98 @@ __global__ void __launch_bounds__(512, 1) tile_onchip_stream(const TileParams p)
     cp_async_wait_all();
 }
 
+// -------------------------------------------------- group-split double-buffered kernel
+// Tiles too large for a cluster's shared memory with double buffering: a group of K
+// co-resident CTAs anywhere on the GPU (cooperative launch; clusters are confined to one
+// GPC, which leaves up to a quarter of the SMs idle at K = 16) owns one tile at a time;
+// CTA k holds slice k (as the cluster kernel) in one of two buffers.  While tile t is
+// written out from one buffer, tile t + groups is fetched into the other with cp.async.
+// In-place rule: a CTA arrives on the group's counter once its slice of a tile is on
+// chip, and stores into that tile only after all K have arrived.  Arrival for the next
+// tile is signalled half-way through the current write-out, so the wait is normally
+// already satisfied (a CTA only arrives for tile i+1 after passing the wait for tile i,
+// hence the cumulative count K*(i+1) identifies tile i).
+__device__ __forceinline__ void group_arrive(uint32_t *ctr) {
+    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
+}
+__device__ __forceinline__ uint64_t global_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+// Spin until the counter reaches `target`.  Co-residency is guaranteed by the cooperative
+// launch; the watchdog turns a violated guarantee into a launch error instead of a hang.
+__device__ __forceinline__ void group_wait(const uint32_t *ctr, uint32_t target) {
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+    if (v >= target) return;
+    const uint64_t t0 = global_ns();
+    do {
+        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+        if (global_ns() - t0 > 20000000000ull) __trap();   // 20 s
+    } while (v < target);
+}
+
+template <int EB>
+__global__ void __launch_bounds__(512, 1) tile_group_db(const TileParams p) {
+    constexpr int V = 16 / EB;
+    extern __shared__ __align__(128) unsigned char smem[];
+    const uint32_t s0 = smem_u32(smem);
+    const uint32_t K = p.K;
+    const uint32_t rank = blockIdx.x % K, gid = blockIdx.x / K, ng = gridDim.x / K;
+    const uint32_t mv = p.m / V, nvr = p.n / V;
+    uint32_t b0, b1, c0, c1, q;
+    if (!p.colsplit) {
+        b0 = (uint32_t)((uint64_t)rank * mv / K);
+        b1 = (uint32_t)((uint64_t)(rank + 1) * mv / K);
+        c0 = 0; c1 = nvr; q = p.q;
+    } else {
+        b0 = 0; b1 = mv;
+        c0 = (uint32_t)((uint64_t)rank * nvr / K);
+        c1 = (uint32_t)((uint64_t)(rank + 1) * nvr / K);
+        q = (c1 - c0) | 1u;
+    }
+    const uint32_t nb = b1 - b0, cvec = c1 - c0;
+    const uint32_t cnt = nb * V * cvec;
+    const uint32_t h = nb / 2;
+    const FastDiv32 divc = make_fastdiv32_dev(cvec);
+    const FastDiv32 div_h = make_fastdiv32_dev(h ? h : 1), div_r = make_fastdiv32_dev(nb - h);
+    uint32_t *ctr = p.gbar + gid * (kGroupCtrStride / 4);
+
+    auto load = [&](const char *g, uint32_t sb) {
+        const char *src = g + ((size_t)b0 * V * nvr + c0) * 16;
+        for (uint32_t e = threadIdx.x; e < cnt; e += blockDim.x) {
+            uint32_t i, j;
+            fdivmod32(e, divc, i, j);
+            cp_async16(sb + (i * q + j) * 16, src + ((size_t)i * nvr + j) * 16);
+        }
+        cp_async_commit();
+    };
+    auto arrive_when_loaded = [&]() {
+        cp_async_wait_all();
+        __syncthreads();
+        if (threadIdx.x == 0) group_arrive(ctr);
+    };
+
+    uint64_t t = gid;
+    if (t < p.count) {
+        load(tile_ptr(p, t), s0);
+        arrive_when_loaded();
+    }
+    for (uint32_t i = 0; t < p.count; t += ng, ++i) {
+        const uint32_t sb = s0 + (i & 1) * p.buf_bytes, sn = s0 + ((i + 1) & 1) * p.buf_bytes;
+        const uint64_t tn = t + ng;
+        if (tn < p.count) load(tile_ptr(p, tn), sn);
+        if (threadIdx.x == 0) group_wait(ctr, K * (i + 1));   // every slice of t on chip
+        __syncthreads();
+        char *g = tile_ptr(p, t);
+        if (h) write_out<EB>(p, sb, g, q, b0, h, div_h, c0, cvec);
+        if (tn < p.count) arrive_when_loaded();
+        write_out<EB>(p, sb + h * V * q * 16, g, q, b0 + h, nb - h, div_r, c0, cvec);
+        __syncthreads();                                      // buffer sb free
+    }
+}
+
 // ------------------------------------------------------------------- generic kernel
 // Any element size and any m x n that fits (Fig. 1 for a CUDA block).  The tile is
 // contiguous, so when it is 16-byte aligned it is loaded with 16-byte vectors; elements
@@ -659,6 +752,10 @@ cudaError_t go(K kern, const TileParams &p, size_t smem, cudaStream_t st, int de
     uint64_t grid = (uint64_t)dp.sms * per_sm;
     if (p.count < grid) grid = p.count;
     if (grid < 1) grid = 1;
+    if (env_int("IPT_DEBUG", 0))
+        fprintf(stderr, "[ipt] tile m=%u n=%u smem=%zu threads=%d per_sm=%d grid=%llu tiles=%llu\n",
+                p.m, p.n, smem, threads, per_sm, (unsigned long long)grid,
+                (unsigned long long)p.count);
     kern<<<(unsigned)grid, threads, smem, st>>>(p);
     note_launch();
     return cudaGetLastError();
@@ -695,9 +792,97 @@ cudaError_t go_cluster(K_ kern, const TileParams &p, size_t smem, int K, cudaStr
     if (clusters < 1) clusters = 1;
     cfg.gridDim = dim3((unsigned)(clusters * K), 1, 1);
     if (env_int("IPT_DEBUG", 0))
-        fprintf(stderr, "[ipt] tile_cluster K=%d smem=%zu threads=%d per_sm=%d maxc=%d clusters=%llu tiles=%llu\n",
-                K, smem, threads, per_sm, maxc, (unsigned long long)clusters, (unsigned long long)p.count);
+        fprintf(stderr, "[ipt] tile_cluster m=%u n=%u K=%d colsplit=%d smem=%zu threads=%d per_sm=%d maxc=%d clusters=%llu tiles=%llu\n",
+                p.m, p.n, K, p.colsplit, smem, threads, per_sm, maxc, (unsigned long long)clusters, (unsigned long long)p.count);
     cudaError_t e = cudaLaunchKernelEx(&cfg, kern, p);
+    note_launch();
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+// Fast-path cluster/group split: column split when the tile has fewer rows than columns
+// (each CTA then writes whole contiguous output rows), else row split.
+static bool fast_colsplit(int64_t A, int64_t B, int eb) {
+    // row-split write segments are ~A*eb/K bytes: only short rows (< 1 KB) favour columns
+    return A < B && A * eb < 1024 && env_int("IPT_TILE_FAST_COLSPLIT", 1);
+}
+
+// Group split (tile_group_db): K CTAs per tile, `groups` tiles in flight, two slice buffers
+// of `slice` bytes per CTA.  Column split when B >= A (the strided side -- reads for a
+// column split, writes for a row split -- then moves B*eb/K-byte rather than A*eb/K-byte
+// pieces; measured 1.1-1.6x either way, tools/tile_big.py).  K minimises waves x (slice + 4 KB barrier allowance); a larger K must win by
+// 3 % (fewer CTAs per barrier, longer pieces).
+static bool group_colsplit(int64_t A, int64_t B) {
+    const long f = env_int("IPT_TILE_GROUP_COLSPLIT", -1);
+    return f >= 0 ? f != 0 : B >= A;
+}
+
+struct GroupCfg {
+    int K = 0, groups = 0;
+    size_t slice = 0;
+    bool colsplit = false;
+};
+
+GroupCfg group_cfg(int64_t A, int64_t B, int eb, uint64_t count, int device) {
+    GroupCfg g;
+    if (!vec_ok(A, B, eb)) return g;
+    const DevProps dp = dev_props(device);
+    const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
+    const int V = 16 / eb;
+    const int64_t mv = A / V, nvr = B / V;
+    const bool cs = group_colsplit(A, B);
+    g.colsplit = cs;
+    const size_t q = fast_q(B, eb);
+    const int kfix = (int)env_int("IPT_TILE_GROUP_K", 0);
+    double best = 1e300;
+    for (int K = 2; K <= dp.sms; ++K) {
+        if (kfix && K != kfix) continue;
+        if ((cs ? nvr : mv) < K) break;
+        size_t slice = cs ? (size_t)A * (size_t)(((nvr + K - 1) / K) | 1) * 16
+                          : (size_t)((mv + K - 1) / K) * V * q * 16;
+        slice = (slice + 127) & ~(size_t)127;
+        if ((long)(2 * slice) > budget) continue;
+        const int64_t groups = std::min<int64_t>(dp.sms / K, (int64_t)std::max<uint64_t>(count, 1));
+        const double waves = (double)((std::max<uint64_t>(count, 1) + groups - 1) / groups);
+        const double cost = waves * ((double)slice + 4096.0);
+        if (cost < best * 0.97) {
+            best = cost;
+            g.K = K;
+            g.groups = (int)groups;
+            g.slice = slice;
+        }
+    }
+    return g;
+}
+
+// Group-split launch: groups x K CTAs, all co-resident (cooperative launch); the arrival
+// counters (workspace, kGroupCtrStride bytes apart) are zeroed on the stream first.
+template <int EB>
+cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g, void *ws,
+                            cudaStream_t st, int device) {
+    if (!ws) return cudaErrorInvalidValue;
+    p.q = fast_q(d.B, d.eb);
+    p.colsplit = g.colsplit ? 1 : 0;
+    p.K = (uint32_t)g.K;
+    p.buf_bytes = (uint32_t)g.slice;
+    p.gbar = (uint32_t *)ws;
+    auto kern = tile_group_db<EB>;
+    cudaError_t e = cudaMemsetAsync(ws, 0, (size_t)g.groups * kGroupCtrStride, st);
+    if (e != cudaSuccess) return e;
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dev_props(device).smem_optin);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(g.groups * g.K), 1, 1);
+    cfg.blockDim = dim3(512, 1, 1);
+    cfg.dynamicSmemBytes = 2 * g.slice;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    if (env_int("IPT_DEBUG", 0))
+        fprintf(stderr, "[ipt] tile_group m=%u n=%u K=%d groups=%d colsplit=%d smem=%zu tiles=%llu\n",
+                p.m, p.n, g.K, g.groups, p.colsplit, 2 * g.slice, (unsigned long long)p.count);
+    e = cudaLaunchKernelEx(&cfg, kern, p);
     note_launch();
     return e != cudaSuccess ? e : cudaGetLastError();
 }
@@ -705,13 +890,7 @@ cudaError_t go_cluster(K_ kern, const TileParams &p, size_t smem, int K, cudaStr
 }  // namespace
 
 // Cluster size for a tile that does not fit one CTA (0 = none): the smallest K in
-// {2, 4, 8} whose row slice fits 113 KB (two CTAs per SM), else the smallest that fits.
-// Fast-path cluster split: column split when the tile has fewer rows than columns (each
-// CTA then writes whole contiguous output rows), else row split.
-static bool fast_colsplit(int64_t A, int64_t B, int eb) {
-    // row-split write segments are ~A*eb/K bytes: only short rows (< 1 KB) favour columns
-    return A < B && A * eb < 1024 && env_int("IPT_TILE_FAST_COLSPLIT", 1);
-}
+// {2, 4, 8, 16} whose slice fits 113 KB (two CTAs per SM), else the smallest that fits.
 
 int tile_cluster_k(int64_t A, int64_t B, int eb, int device) {
     if (!vec_ok(A, B, eb) || !env_int("IPT_TILE_CLUSTER", 1)) return 0;
@@ -777,10 +956,37 @@ int tile_generic_cluster_k(int64_t A, int64_t B, int eb, int device) {
     return 0;
 }
 
+// Group split instead of a cluster (measured, tools/tile_big.py): when no cluster fits, when
+// the cluster's slices need one CTA per SM (streaming kernel), and for K >= 8 (clusters of
+// 8 and 16 strand SMs: 14 co-resident 16-CTA clusters at two CTAs per SM, 7 at one).
+// Clusters of 2 or 4 with two CTAs per SM are as fast or faster and need no workspace.
+bool tile_group_split(int64_t A, int64_t B, int eb, int device) {
+    if (!vec_ok(A, B, eb) || !env_int("IPT_TILE_GROUP_SPLIT", 1)) return false;
+    const DevProps dp = dev_props(device);
+    const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
+    if ((long)fast_smem(A, B, eb) <= budget) return false;
+    const int K = tile_cluster_k(A, B, eb, device);
+    if (K && K < 8) {
+        const int V = 16 / eb;
+        const size_t slice = fast_colsplit(A, B, eb)
+            ? (size_t)A * (size_t)((((B / V) + K - 1) / K) | 1) * 16
+            : (size_t)(((A / V) + K - 1) / K) * V * (size_t)fast_q(B, eb) * 16;
+        if (slice <= 113 * 1024) return false;
+    }
+    return group_cfg(A, B, eb, (uint64_t)dp.sms, device).K != 0;
+}
+
+int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups) {
+    const GroupCfg g = group_cfg(A, B, eb, count, device);
+    if (groups) *groups = g.groups;
+    return g.K;
+}
+
 int tile_onchip_path(int64_t A, int64_t B, int eb, int device) {
     DevProps dp = dev_props(device);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
     if (vec_ok(A, B, eb) && (long)fast_smem(A, B, eb) <= budget) return 2;
+    if (tile_group_split(A, B, eb, device)) return 5;
     if (tile_cluster_k(A, B, eb, device)) return 3;
     if ((long)generic_smem(A, B, eb) > budget && tile_generic_cluster_k(A, B, eb, device)) return 4;
     if ((long)generic_smem(A, B, eb) <= budget && A * B < (1ll << 31)) return 1;
@@ -791,7 +997,7 @@ bool tile_onchip_fits(int64_t A, int64_t B, int eb, int device) {
     return tile_onchip_path(A, B, eb, device) != 0;
 }
 
-cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) {
+cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, int device) {
     DevProps dp = dev_props(device);
     TileParams p{};
     p.base = d.base;
@@ -841,6 +1047,14 @@ cudaError_t launch_tile_onchip(const StageDesc &d, cudaStream_t st, int device) 
                 case 16: return big ? go(tile_onchip_ldg<16, 16, 1>, p, smem, st, device)
                                     : go(tile_onchip_ldg<16, 8>, p, smem, st, device);
             }
+        }
+    }
+    if (fast_ok(d) && tile_group_split(d.A, d.B, d.eb, device)) {
+        const GroupCfg g = group_cfg(d.A, d.B, d.eb, p.count, device);
+        switch (d.eb) {
+            case 4: return launch_group_db<4>(d, p, g, ws, st, device);
+            case 8: return launch_group_db<8>(d, p, g, ws, st, device);
+            case 16: return launch_group_db<16>(d, p, g, ws, st, device);
         }
     }
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) > budget) {

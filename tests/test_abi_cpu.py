@@ -148,7 +148,8 @@ def test_plan_prefers_vector_tiles_on_large_f32():
         assert p.n * 4 >= 256 and p.m * 4 >= 256
         assert p.n * 4 % 16 == 0 and p.m * 4 % 16 == 0     # 16-byte vector super-elements
         assert ipt.VARIANTS[p.variant[1]] == "tile_onchip"
-        assert p.n_stages == 3
+        # 3 stages, or 2 when a whole M x n (m x N) panel fits a group of CTAs on chip
+        assert p.n_stages == 3 or (p.n_stages == 2 and (p.m == M or p.n == N))
     # panel plans (stages 2+3 fused, m = M) where the whole M x n panel fits a cluster
     p = ipt.plan(7200, 18000, 4)
     assert p.n_stages >= 2 and ipt.VARIANTS[p.variant[1]] == "tile_onchip"

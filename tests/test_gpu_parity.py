@@ -281,6 +281,23 @@ def test_batched_with_stride():
     assert np.array_equal(to_np(t, 4), ref)
 
 
+def test_batched_plan_events():
+    count, M, N = 5, 720, 1800
+    p = ipt.plan(M, N, 4, device=0)
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+    for e in evs:
+        e.record()
+    a = seeded.values_np(np.arange(count * M * N), 4)
+    t = to_dev(a, 4)
+    ipt.transpose_batched_(t, count, M, N, plan_=p, events=evs)
+    torch.cuda.synchronize()
+    ref = a.copy()
+    for i in range(count):
+        oracle.transpose_inplace(ref[i * M * N:(i + 1) * M * N], M, N)
+    assert np.array_equal(to_np(t, 4), ref)
+    assert all(evs[i].elapsed_time(evs[i + 1]) >= 0 for i in range(3))
+
+
 # ------------------------------------------------------------------ race stress (T6)
 def test_stress_varied_occupancy(monkeypatch):
     """Repeat with different persistent-grid sizes and walker shapes so chains
@@ -391,9 +408,11 @@ def test_transpose_host_queues(queues):
 # ------------------------------------------------- cluster-split tiles (> 227 KB)
 @pytest.mark.parametrize("eb,batch,A,B", [(4, 3, 512, 512), (4, 2, 7200 // 4, 60), (4, 5, 640, 600),
                                           (8, 3, 400, 400), (16, 2, 256, 256), (4, 7, 960, 400)])
-def test_ipt_010_cluster_tiles(eb, batch, A, B):
+@pytest.mark.parametrize("split", ["0", "1"])
+def test_ipt_010_cluster_tiles(monkeypatch, split, eb, batch, A, B):
     """Tiles larger than one CTA's shared memory are split over a thread-block cluster
     (one barrier.cluster per tile); bit-exact vs the oracle."""
+    monkeypatch.setenv("IPT_TILE_GROUP_SPLIT", split)   # cluster vs group split
     a = gen(batch * A * B, eb)
     t = to_dev(a, eb)
     ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
@@ -470,8 +489,10 @@ def test_layout_marshaling(M, N, m):
 
 
 @pytest.mark.parametrize("eb,batch,A,B", [(4, 2, 1800, 240), (8, 3, 902, 100), (4, 2, 3004, 128)])
-def test_ipt_010_cluster_uneven_slices(eb, batch, A, B):
+@pytest.mark.parametrize("split", ["0", "1"])
+def test_ipt_010_cluster_uneven_slices(monkeypatch, split, eb, batch, A, B):
     """16-byte cluster path with row slices of unequal length (multiples of V rows)."""
+    monkeypatch.setenv("IPT_TILE_GROUP_SPLIT", split)   # cluster vs group split
     a = gen(batch * A * B, eb)
     t = to_dev(a, eb)
     ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
@@ -479,8 +500,9 @@ def test_ipt_010_cluster_uneven_slices(eb, batch, A, B):
 
 
 @pytest.mark.parametrize("eb,batch,A,B", [(4, 2, 7200, 120), (4, 1, 9998, 64)])
-def test_ipt_010_cluster16(eb, batch, A, B):
+def test_ipt_010_cluster16(monkeypatch, eb, batch, A, B):
     """Non-portable 16-CTA clusters (panels up to 16 x 227 KB)."""
+    monkeypatch.setenv("IPT_TILE_GROUP_SPLIT", "0")
     a = gen(batch * A * B, eb)
     t = to_dev(a, eb)
     ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
@@ -489,9 +511,11 @@ def test_ipt_010_cluster16(eb, batch, A, B):
 
 @pytest.mark.parametrize("eb,batch,A,B", [(4, 2, 120, 7200), (8, 2, 64, 2000), (16, 2, 32, 3000),
                                           (4, 3, 256, 1000)])
-def test_ipt_010_cluster_column_split_fast(eb, batch, A, B):
+@pytest.mark.parametrize("split", ["0", "1"])
+def test_ipt_010_cluster_column_split_fast(monkeypatch, split, eb, batch, A, B):
     """16-byte cluster path, fewer rows than columns: each CTA owns a range of 16-byte
     columns and writes whole contiguous output rows."""
+    monkeypatch.setenv("IPT_TILE_GROUP_SPLIT", split)   # cluster vs group split
     a = gen(batch * A * B, eb)
     t = to_dev(a, eb)
     ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
@@ -528,9 +552,10 @@ def test_transpose_host_async_two_streams():
 
 @pytest.mark.parametrize("eb,batch,A,B", [(4, 5, 256, 200), (8, 4, 120, 200), (16, 3, 100, 120),
                                           (4, 3, 7200, 120), (4, 7, 1800, 160), (8, 2, 1000, 96)])
-def test_ipt_010_streaming_slices(eb, batch, A, B):
+def test_ipt_010_streaming_slices(monkeypatch, eb, batch, A, B):
     """One CTA per SM (slices > 113 KB): write-out of tile t overlapped with the cp.async
     refill of tile t+1, group by group."""
+    monkeypatch.setenv("IPT_TILE_GROUP_SPLIT", "0")
     a = gen(batch * A * B, eb)
     t = to_dev(a, eb)
     ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
@@ -595,3 +620,59 @@ def test_concurrent_streams_internal_workspace():
     torch.cuda.synchronize()
     for t, ref in zip(ts, refs):
         assert np.array_equal(to_np(t, 4), ref)
+
+
+# ------------------------------------------ group-split tiles (co-resident CTA groups)
+@pytest.mark.parametrize("eb,batch,A,B", [(4, 3, 120, 7200), (4, 2, 7200, 120), (4, 2, 60, 7200),
+                                          (4, 3, 180, 7200), (8, 2, 400, 800), (16, 2, 300, 400),
+                                          (4, 1, 1024, 1024), (4, 1, 128, 16384), (8, 1, 1000, 1000),
+                                          (4, 5, 720, 720)])
+def test_ipt_010_group_split(eb, batch, A, B):
+    """Tiles split over a co-resident group of K CTAs (cooperative launch, software barrier
+    per tile, double-buffered slices) -- including tiles beyond 16 x 227 KB clusters."""
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)
+
+
+@pytest.mark.parametrize("K", ["16", "17", "31", "37", "75", "148"])
+@pytest.mark.parametrize("split", ["0", "1"])
+def test_ipt_010_group_forced_sizes(monkeypatch, K, split):
+    """Any group size (not only cluster sizes), uneven slices, both split directions."""
+    monkeypatch.setenv("IPT_TILE_GROUP_K", K)
+    monkeypatch.setenv("IPT_TILE_GROUP_COLSPLIT", split)
+    batch, A, B = 7, 600, 1200
+    a = gen(batch * A * B, 4)
+    t = to_dev(a, 4)
+    ipt.ipt_010_(t, batch, A, B)
+    assert np.array_equal(to_np(t, 4), oracle_P(a.copy(), batch, A, B, 1, 4)), (K, split)
+
+
+_CONCURRENT_GROUPS = r"""
+import sys, torch
+sys.path.insert(0, sys.argv[1])
+import paper_conf_ppopp_sunggggh14_b200 as ipt
+shapes = [(3, 120, 7200), (2, 7200, 120), (1, 1024, 1024), (4, 720, 720)]
+sts = [torch.cuda.Stream() for _ in shapes]
+ts = [torch.randint(0, 2**31 - 1, (b * A * B,), dtype=torch.int32, device="cuda") for (b, A, B) in shapes]
+refs = [t.clone() for t in ts]
+for rep in range(40):
+    for (b, A, B), t, s in zip(shapes, ts, sts):
+        x, y = (A, B) if rep % 2 == 0 else (B, A)
+        ipt.ipt_010_(t, b, x, y, stream=s)
+torch.cuda.synchronize()
+assert all(torch.equal(t, r) for t, r in zip(ts, refs))
+print("ok")
+"""
+
+
+def test_group_split_concurrent_streams():
+    """Cooperative group-split launches on four streams at once (each with its own
+    counters) complete and are exact; run in a child with a deadline so a co-residency
+    failure cannot hang the suite."""
+    import subprocess, sys, os
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", _CONCURRENT_GROUPS, root], capture_output=True,
+                       text=True, timeout=180)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]

@@ -1,3 +1,4 @@
 cd $GRAFT_REPO_ROOT
-export SHAPES="[(7200,120),(10000,64),(120,7200),(256,200)]"
-for g in 0 8 16 32 0; do IPT_TILE_GROUP=$g timeout 300 python tools/tile_sweep.py | sed "s/^/GB=$g /" >> gpurun_out/tile_sweep.log 2>&1; done
+export SHAPES="${SHAPES:-[(120,7200),(7200,120),(60,12800),(12800,60),(64,10000),(10000,64),(32,20000),(20000,32),(256,256)]}"
+export VARIANTS="${VARIANTS:-[{\"IPT_DEBUG\":1}]}"
+timeout 900 python tools/tile_big.py > gpurun_out/tile_big.txt 2>&1

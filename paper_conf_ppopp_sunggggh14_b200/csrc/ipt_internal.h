@@ -89,11 +89,13 @@ bool tile_onchip_fits(int64_t A, int64_t B, int eb, int device);
 // 0: does not fit, 1: generic element path, 2: 16-byte path in one CTA,
 // 3: 16-byte path split over a thread-block cluster (tile_cluster_k CTAs),
 // 4: element path split over a thread-block cluster,
-// 5: 16-byte path split over a co-resident group of CTAs (double-buffered slices)
+// 5: 16-byte path split over a co-resident group of CTAs (double-buffered slices),
+// 6: element path (4/8-byte elements) split over a co-resident group of CTAs
 int tile_onchip_path(int64_t A, int64_t B, int eb, int device);
 int tile_cluster_k(int64_t A, int64_t B, int eb, int device);
 int tile_generic_cluster_k(int64_t A, int64_t B, int eb, int device);
 bool tile_group_split(int64_t A, int64_t B, int eb, int device);
+bool tile_group_generic_split(int64_t A, int64_t B, int eb, int device);
 // Group split of `count` tiles: CTAs per tile (0 = does not fit) and groups in flight.
 int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups);
 // Workspace of a tile stage: the group split's arrival counters (one per group,

@@ -533,6 +533,107 @@ __global__ void __launch_bounds__(512, 1) tile_group_db(const TileParams p) {
     }
 }
 
+// ------------------------------------------------- group-split element-path kernel
+// Tiles whose sides are not multiples of 16/elem (e.g. 64 x 9998 or 14803 x 32 floats),
+// 4- and 8-byte elements, over a CTA group as tile_group_db.  A slice is a set of row
+// pieces: rows [r0, r1) x columns [c0, c1) (row split: all columns; column split: all
+// rows).  Each piece is fetched with cp.async as the 16-byte vectors covering it, kept at
+// its global 16-byte phase (sh = first element's offset in its vector) in a shared row of
+// Q vectors (Q odd).  Write-out: a warp takes 32 consecutive rows x PV consecutive
+// columns; each lane reads the two vectors holding its PV elements, aligns them with a
+// select network, and the warp stores PV runs of 32 consecutive output elements.
+template <int EB>
+__global__ void __launch_bounds__(512, 1) tile_group_generic(const TileParams p) {
+    constexpr uint32_t PV = 16 / EB;
+    using E = typename Elem<EB>::T;
+    extern __shared__ __align__(128) unsigned char smem[];
+    const uint32_t s0 = smem_u32(smem);
+    const uint32_t K = p.K;
+    const uint32_t rank = blockIdx.x % K, gid = blockIdx.x / K, ng = gridDim.x / K;
+    uint32_t r0, r1, c0, c1;
+    if (p.colsplit) {
+        r0 = 0; r1 = p.m;
+        c0 = (uint32_t)((uint64_t)rank * p.n / K);
+        c1 = (uint32_t)((uint64_t)(rank + 1) * p.n / K);
+    } else {
+        c0 = 0; c1 = p.n;
+        r0 = (uint32_t)((uint64_t)rank * p.m / K);
+        r1 = (uint32_t)((uint64_t)(rank + 1) * p.m / K);
+    }
+    const uint32_t rows = r1 - r0, L = c1 - c0, Q = p.q;
+    const uint32_t QV = (L + 2 * PV - 2) / PV;            // covering vectors, worst phase
+    const FastDiv32 divq = make_fastdiv32_dev(QV);
+    const uint32_t nrb = (rows + 31) / 32, ncb = (L + PV - 1) / PV;
+    const uint32_t ntask = nrb * ncb;
+    const FastDiv32 divrb = make_fastdiv32_dev(nrb);
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+    uint32_t *ctr = p.gbar + gid * (kGroupCtrStride / 4);
+
+    auto load = [&](const char *g, uint32_t sb) {
+        const uint32_t cnt = rows * QV;
+        for (uint32_t e = threadIdx.x; e < cnt; e += blockDim.x) {
+            uint32_t i, j;
+            fdivmod32(e, divq, i, j);
+            const uintptr_t a = (uintptr_t)(g + ((uint64_t)(r0 + i) * p.n + c0) * EB);
+            const uint32_t sh = (uint32_t)(a & 15) / EB;
+            if (j * PV < sh + L) cp_async16(sb + (i * Q + j) * 16, (const void *)((a & ~(uintptr_t)15) + j * 16));
+        }
+        cp_async_commit();
+    };
+    auto write = [&](char *g, uint32_t sb, uint32_t task0, uint32_t task1) {
+        for (uint32_t task = task0 + warp; task < task1; task += nw) {
+            uint32_t cb, rb;
+            fdivmod32(task, divrb, cb, rb);
+            const uint32_t i = rb * 32 + lane, c = cb * PV;
+            E x[2 * PV];
+            if (i < rows) {
+                const uintptr_t a = (uintptr_t)(g + ((uint64_t)(r0 + i) * p.n + c0) * EB);
+                const uint32_t w = (uint32_t)(a & 15) / EB + c;
+                const uint32_t v = w / PV, o = w % PV;
+                E ex[PV], ey[PV];
+                unpack<EB>(lds128(sb + (i * Q + v) * 16), ex);
+                unpack<EB>(lds128(sb + (i * Q + v + 1) * 16), ey);
+#pragma unroll
+                for (uint32_t k = 0; k < PV; ++k) { x[k] = ex[k]; x[PV + k] = ey[k]; }
+#pragma unroll
+                for (uint32_t sft = 1; sft < PV; sft <<= 1) {   // x[k] <- x[k + o]
+                    const bool f = (o & sft) != 0;
+#pragma unroll
+                    for (uint32_t k = 0; k + sft < 2 * PV; ++k) x[k] = f ? x[k + sft] : x[k];
+                }
+            }
+#pragma unroll
+            for (uint32_t k = 0; k < PV; ++k) {
+                if (i < rows && c + k < L)
+                    *reinterpret_cast<E *>(g + ((uint64_t)(c0 + c + k) * p.m + r0 + i) * EB) = x[k];
+            }
+        }
+    };
+    auto arrive_when_loaded = [&]() {
+        cp_async_wait_all();
+        __syncthreads();
+        if (threadIdx.x == 0) group_arrive(ctr);
+    };
+
+    uint64_t t = gid;
+    if (t < p.count) {
+        load(tile_ptr(p, t), s0);
+        arrive_when_loaded();
+    }
+    for (uint32_t it = 0; t < p.count; t += ng, ++it) {
+        const uint32_t sb = s0 + (it & 1) * p.buf_bytes, sn = s0 + ((it + 1) & 1) * p.buf_bytes;
+        const uint64_t tn = t + ng;
+        if (tn < p.count) load(tile_ptr(p, tn), sn);
+        if (threadIdx.x == 0) group_wait(ctr, K * (it + 1));
+        __syncthreads();
+        char *g = tile_ptr(p, t);
+        write(g, sb, 0, ntask / 2);
+        if (tn < p.count) arrive_when_loaded();
+        write(g, sb, ntask / 2, ntask);
+        __syncthreads();
+    }
+}
+
 // ------------------------------------------------------------------- generic kernel
 // Any element size and any m x n that fits (Fig. 1 for a CUDA block).  The tile is
 // contiguous, so when it is 16-byte aligned it is loaded with 16-byte vectors; elements
@@ -854,18 +955,57 @@ GroupCfg group_cfg(int64_t A, int64_t B, int eb, uint64_t count, int device) {
     return g;
 }
 
+// Element-path group split: slices of row pieces (see tile_group_generic), one padding
+// vector per buffer (the aligner may read one vector past the last row).
+GroupCfg group_cfg_generic(int64_t A, int64_t B, int eb, uint64_t count, int device) {
+    GroupCfg g;
+    if (eb != 4 && eb != 8) return g;
+    const DevProps dp = dev_props(device);
+    const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
+    const int PV = 16 / eb;
+    const bool cs = group_colsplit(A, B);
+    g.colsplit = cs;
+    const int kfix = (int)env_int("IPT_TILE_GROUP_K", 0);
+    double best = 1e300;
+    for (int K = 2; K <= dp.sms; ++K) {
+        if (kfix && K != kfix) continue;
+        if ((cs ? B : A) < (int64_t)K * (cs ? PV : 1)) break;
+        const int64_t L = cs ? (B + K - 1) / K : B;
+        const int64_t rows = cs ? A : (A + K - 1) / K;
+        const int64_t Q = ((L + 2 * PV - 2) / PV) | 1;
+        size_t slice = (size_t)(rows * Q + 1) * 16;
+        slice = (slice + 127) & ~(size_t)127;
+        if ((long)(2 * slice) > budget) continue;
+        const int64_t groups = std::min<int64_t>(dp.sms / K, (int64_t)std::max<uint64_t>(count, 1));
+        const double waves = (double)((std::max<uint64_t>(count, 1) + groups - 1) / groups);
+        const double cost = waves * ((double)slice + 4096.0);
+        if (cost < best * 0.97) {
+            best = cost;
+            g.K = K;
+            g.groups = (int)groups;
+            g.slice = slice;
+        }
+    }
+    return g;
+}
+
 // Group-split launch: groups x K CTAs, all co-resident (cooperative launch); the arrival
 // counters (workspace, kGroupCtrStride bytes apart) are zeroed on the stream first.
-template <int EB>
+template <int EB, bool GENERIC>
 cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g, void *ws,
                             cudaStream_t st, int device) {
-    if (!ws) return cudaErrorInvalidValue;
-    p.q = fast_q(d.B, d.eb);
+    if (!ws || !g.K) return cudaErrorInvalidValue;
+    if (GENERIC) {
+        const int64_t L = g.colsplit ? (d.B + g.K - 1) / g.K : d.B;
+        p.q = (uint32_t)(((L + 2 * (16 / EB) - 2) / (16 / EB)) | 1);
+    } else {
+        p.q = fast_q(d.B, d.eb);
+    }
     p.colsplit = g.colsplit ? 1 : 0;
     p.K = (uint32_t)g.K;
     p.buf_bytes = (uint32_t)g.slice;
     p.gbar = (uint32_t *)ws;
-    auto kern = tile_group_db<EB>;
+    auto kern = GENERIC ? tile_group_generic<EB> : tile_group_db<EB>;
     cudaError_t e = cudaMemsetAsync(ws, 0, (size_t)g.groups * kGroupCtrStride, st);
     if (e != cudaSuccess) return e;
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dev_props(device).smem_optin);
@@ -880,8 +1020,9 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     if (env_int("IPT_DEBUG", 0))
-        fprintf(stderr, "[ipt] tile_group m=%u n=%u K=%d groups=%d colsplit=%d smem=%zu tiles=%llu\n",
-                p.m, p.n, g.K, g.groups, p.colsplit, 2 * g.slice, (unsigned long long)p.count);
+        fprintf(stderr, "[ipt] tile_group%s m=%u n=%u K=%d groups=%d colsplit=%d smem=%zu tiles=%llu\n",
+                GENERIC ? "_generic" : "", p.m, p.n, g.K, g.groups, p.colsplit, 2 * g.slice,
+                (unsigned long long)p.count);
     e = cudaLaunchKernelEx(&cfg, kern, p);
     note_launch();
     return e != cudaSuccess ? e : cudaGetLastError();
@@ -976,8 +1117,17 @@ bool tile_group_split(int64_t A, int64_t B, int eb, int device) {
     return group_cfg(A, B, eb, (uint64_t)dp.sms, device).K != 0;
 }
 
+// Element path over a CTA group (4- and 8-byte elements) when the tile needs more than
+// 113 KB of one CTA (measured faster than the single-CTA and cluster element kernels).
+bool tile_group_generic_split(int64_t A, int64_t B, int eb, int device) {
+    if ((eb != 4 && eb != 8) || !env_int("IPT_TILE_GROUP_GENERIC", 1)) return false;
+    if ((size_t)generic_smem(A, B, eb) <= 113 * 1024) return false;
+    return group_cfg_generic(A, B, eb, (uint64_t)dev_props(device).sms, device).K != 0;
+}
+
 int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups) {
-    const GroupCfg g = group_cfg(A, B, eb, count, device);
+    const GroupCfg g = vec_ok(A, B, eb) ? group_cfg(A, B, eb, count, device)
+                                        : group_cfg_generic(A, B, eb, count, device);
     if (groups) *groups = g.groups;
     return g.K;
 }
@@ -988,6 +1138,7 @@ int tile_onchip_path(int64_t A, int64_t B, int eb, int device) {
     if (vec_ok(A, B, eb) && (long)fast_smem(A, B, eb) <= budget) return 2;
     if (tile_group_split(A, B, eb, device)) return 5;
     if (tile_cluster_k(A, B, eb, device)) return 3;
+    if (!vec_ok(A, B, eb) && tile_group_generic_split(A, B, eb, device)) return 6;
     if ((long)generic_smem(A, B, eb) > budget && tile_generic_cluster_k(A, B, eb, device)) return 4;
     if ((long)generic_smem(A, B, eb) <= budget && A * B < (1ll << 31)) return 1;
     return 0;
@@ -1052,9 +1203,16 @@ cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, in
     if (fast_ok(d) && tile_group_split(d.A, d.B, d.eb, device)) {
         const GroupCfg g = group_cfg(d.A, d.B, d.eb, p.count, device);
         switch (d.eb) {
-            case 4: return launch_group_db<4>(d, p, g, ws, st, device);
-            case 8: return launch_group_db<8>(d, p, g, ws, st, device);
-            case 16: return launch_group_db<16>(d, p, g, ws, st, device);
+            case 4: return launch_group_db<4, false>(d, p, g, ws, st, device);
+            case 8: return launch_group_db<8, false>(d, p, g, ws, st, device);
+            case 16: return launch_group_db<16, false>(d, p, g, ws, st, device);
+        }
+    }
+    if (!fast_ok(d) && tile_group_generic_split(d.A, d.B, d.eb, device)) {
+        const GroupCfg g = group_cfg_generic(d.A, d.B, d.eb, p.count, device);
+        switch (d.eb) {
+            case 4: return launch_group_db<4, true>(d, p, g, ws, st, device);
+            case 8: return launch_group_db<8, true>(d, p, g, ws, st, device);
         }
     }
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) > budget) {

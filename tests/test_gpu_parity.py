@@ -676,3 +676,40 @@ def test_group_split_concurrent_streams():
     r = subprocess.run([sys.executable, "-c", _CONCURRENT_GROUPS, root], capture_output=True,
                        text=True, timeout=180)
     assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
+
+
+@pytest.mark.parametrize("eb,batch,A,B", [(4, 2, 64, 9998), (4, 2, 9998, 64), (4, 2, 113, 8192),
+                                          (4, 1, 14803, 32), (4, 1, 14803, 128), (8, 2, 3001, 61),
+                                          (8, 2, 61, 3001), (4, 3, 301, 257), (4, 2, 7, 40001),
+                                          (4, 3, 1999, 31), (8, 1, 2999, 257)])
+def test_ipt_010_group_split_element_path(eb, batch, A, B):
+    """Element-path tiles (sides not multiples of 16/elem) over a CTA group: row pieces
+    fetched at their global 16-byte phase and realigned in registers on write-out."""
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B)
+
+
+@pytest.mark.parametrize("K", ["2", "5", "37", "148"])
+@pytest.mark.parametrize("split", ["0", "1"])
+def test_ipt_010_group_element_forced_sizes(monkeypatch, K, split):
+    monkeypatch.setenv("IPT_TILE_GROUP_K", K)
+    monkeypatch.setenv("IPT_TILE_GROUP_COLSPLIT", split)
+    batch, A, B = 5, 601, 1203
+    a = gen(batch * A * B, 4)
+    t = to_dev(a, 4)
+    ipt.ipt_010_(t, batch, A, B)
+    assert np.array_equal(to_np(t, 4), oracle_P(a.copy(), batch, A, B, 1, 4)), (K, split)
+
+
+def test_ipt_010_group_element_misaligned_base():
+    """A 16-byte-vectorisable tile at a base that is only 4-byte aligned takes the
+    element-path group kernel (any phase)."""
+    batch, A, B = 3, 400, 800
+    a = gen(batch * A * B + 1, 4)
+    t = to_dev(a, 4)
+    ipt.ipt_010_(t[1:], batch, A, B)
+    ref = a.copy()
+    ref[1:] = oracle_P(a[1:].copy(), batch, A, B, 1, 4)
+    assert np.array_equal(to_np(t, 4), ref)

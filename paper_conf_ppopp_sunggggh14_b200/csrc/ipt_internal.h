@@ -98,8 +98,8 @@ bool tile_group_split(int64_t A, int64_t B, int eb, int device);
 bool tile_group_generic_split(int64_t A, int64_t B, int eb, int device);
 // Group split of `count` tiles: CTAs per tile (0 = does not fit) and groups in flight.
 int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups);
-// Workspace of a tile stage: the group split's arrival counters (one per group,
-// kGroupCtrStride bytes apart, at most 256 groups).  `ws` may be NULL for the other paths.
+// Workspace of a tile stage: the group split's arrival counters (one per group and slice
+// buffer, kGroupCtrStride bytes apart, at most 256).  `ws` may be NULL for the other paths.
 constexpr uint32_t kGroupCtrStride = 32;
 constexpr size_t kTileWsBytes = 256 * kGroupCtrStride;
 cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, int device);

@@ -110,15 +110,20 @@ __device__ __forceinline__ void sts128(uint32_t saddr, const uint4 &v) {
 // block rows [bi0, bi0 + mvp) x block columns [bj0, bj0 + nbj) of the tile (V x V blocks):
 // buffer row bil*V + r, 16-byte column bjl (pitch q) holds tile row (bi0+bil)*V + r,
 // columns (bj0+bjl)*V .. +V-1.  Whole tile for one CTA; a row or column slice per cluster CTA.
-template <int EB>
+struct NoProbe {
+    __device__ void operator()() const {}
+};
+
+template <int EB, typename Probe = NoProbe>
 __device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, char *g, uint32_t q,
                                           uint32_t bi0, uint32_t mvp, const FastDiv32 &divmvp,
-                                          uint32_t bj0, uint32_t nbj) {
+                                          uint32_t bj0, uint32_t nbj, Probe probe = Probe()) {
     constexpr int V = 16 / EB;
     constexpr int ROT = (V >= 8) ? 1 : 8 / V;   // lanes sharing one rotation
     using E = typename Elem<EB>::T;
     const uint32_t nblk = mvp * nbj;
     for (uint32_t blk = threadIdx.x; blk < nblk; blk += blockDim.x) {
+        probe();
         uint32_t bjl, bil;
         fdivmod32(blk, divmvp, bjl, bil);
         const uint32_t bi = bi0 + bil, bj = bj0 + bjl;
@@ -473,13 +478,101 @@ __device__ __forceinline__ void group_wait(const uint32_t *ctr, uint32_t target)
     } while (v < target);
 }
 
+constexpr uint32_t kGroupMaxBuf = 4;
+
+// Ring of p.nbuf slice buffers shared by the group kernels.  Iteration j of a group
+// handles tile gid + j*groups in buffer j % nbuf; the loads of tile j + nbuf - 1 are
+// issued at the start of iteration j, so a slice has nbuf - 1 write-outs to land.  Its
+// cp.async copies arrive on the buffer's mbarrier (cp.async.mbarrier.arrive: no warp
+// stalls on them); thread 0 probes the barriers while writing and signals the group, in
+// tile order, once each slice has landed.  One counter per (group, buffer): a CTA arrives
+// for tile j + nbuf only after finishing tile j, i.e. after all K arrivals for tile j, so
+// counter j % nbuf reaching K * (j / nbuf + 1) means exactly "every slice of tile j is on
+// chip".
+struct GroupPipe {
+    uint64_t *mbar;     // nbuf mbarriers in shared memory
+    uint32_t *ctr;      // this group's counters, kGroupCtrStride bytes apart
+    uint32_t K, nbuf;
+    uint32_t na = 0;    // thread 0: next iteration to arrive for
+    __device__ void init() {
+        if (threadIdx.x == 0) {
+            for (uint32_t b = 0; b < nbuf; ++b) mbar_init(&mbar[b], blockDim.x);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+        __syncthreads();
+    }
+    __device__ uint32_t *slot(uint32_t j) const { return ctr + (j % nbuf) * (kGroupCtrStride / 4); }
+    __device__ void issued(uint32_t j) { cp_async_mbar_arrive(&mbar[j % nbuf]); }
+    __device__ bool landed(uint32_t j) { return mbar_test_wait(&mbar[j % nbuf], (j / nbuf) & 1); }
+    __device__ void wait_landed(uint32_t j) { mbar_wait(&mbar[j % nbuf], (j / nbuf) & 1); }
+    __device__ void probe(uint32_t limit) {          // thread 0
+        while (na < limit && landed(na)) group_arrive(slot(na++));
+    }
+    __device__ void force(uint32_t j) {              // thread 0: arrivals up to j
+        while (na <= j) {
+            wait_landed(na);
+            group_arrive(slot(na++));
+        }
+    }
+    __device__ void wait_group(uint32_t j) { group_wait(slot(j), K * (j / nbuf + 1)); }
+};
+
+// Main loop of a group kernel: load(tile pointer, buffer address) issues the cp.async
+// copies of one slice; write(tile pointer, buffer address, part, parts, probe) writes part
+// `part` of `parts` of one out, calling probe() now and then.  MIDSYNC: instead of
+// probing, the CTA waits for the next slice half-way through the write-out and then
+// arrives (measured faster for the element-path kernel, slower for the 16-byte one).
+template <bool MIDSYNC, typename Load, typename Write>
+__device__ __forceinline__ void group_loop(const TileParams &p, uint32_t s0, uint64_t *mbar,
+                                           Load load, Write write) {
+    const uint32_t K = p.K, gid = blockIdx.x / K, ng = gridDim.x / K;
+    GroupPipe pipe;
+    pipe.mbar = mbar;
+    pipe.ctr = p.gbar + gid * p.nbuf * (kGroupCtrStride / 4);
+    pipe.K = K;
+    pipe.nbuf = p.nbuf;
+    pipe.init();
+    const uint32_t nt = gid < p.count ? (uint32_t)((p.count - gid + ng - 1) / ng) : 0;
+    auto issue = [&](uint32_t j) {
+        load(tile_ptr(p, gid + (uint64_t)j * ng), s0 + (j % p.nbuf) * p.buf_bytes);
+        pipe.issued(j);
+    };
+    for (uint32_t j = 0; j + 1 < p.nbuf && j < nt; ++j) issue(j);
+    for (uint32_t i = 0; i < nt; ++i) {
+        const uint32_t jn = i + p.nbuf - 1;
+        if (jn < nt) issue(jn);
+        const uint32_t lim = min(nt, jn + 1);
+        pipe.wait_landed(i);                         // own slice of tile i on chip
+        if (threadIdx.x == 0) {
+            pipe.force(i);
+            pipe.wait_group(i);                      // every slice of tile i on chip
+        }
+        __syncthreads();
+        char *g = tile_ptr(p, gid + (uint64_t)i * ng);
+        const uint32_t sb = s0 + (i % p.nbuf) * p.buf_bytes;
+        if (MIDSYNC) {
+            auto none = []() {};
+            write(g, sb, 0, 2, none);
+            if (jn < nt) {
+                pipe.wait_landed(jn);
+                __syncthreads();
+                if (threadIdx.x == 0) pipe.force(jn);
+            }
+            write(g, sb, 1, 2, none);
+        } else {
+            write(g, sb, 0, 1, [&]() { if (threadIdx.x == 0) pipe.probe(lim); });
+        }
+        __syncthreads();                             // buffer i % nbuf free
+    }
+}
+
 template <int EB>
 __global__ void __launch_bounds__(512, 1) tile_group_db(const TileParams p) {
     constexpr int V = 16 / EB;
     extern __shared__ __align__(128) unsigned char smem[];
     const uint32_t s0 = smem_u32(smem);
     const uint32_t K = p.K;
-    const uint32_t rank = blockIdx.x % K, gid = blockIdx.x / K, ng = gridDim.x / K;
+    const uint32_t rank = blockIdx.x % K;
     const uint32_t mv = p.m / V, nvr = p.n / V;
     uint32_t b0, b1, c0, c1, q;
     if (!p.colsplit) {
@@ -494,43 +587,20 @@ __global__ void __launch_bounds__(512, 1) tile_group_db(const TileParams p) {
     }
     const uint32_t nb = b1 - b0, cvec = c1 - c0;
     const uint32_t cnt = nb * V * cvec;
-    const uint32_t h = nb / 2;
-    const FastDiv32 divc = make_fastdiv32_dev(cvec);
-    const FastDiv32 div_h = make_fastdiv32_dev(h ? h : 1), div_r = make_fastdiv32_dev(nb - h);
-    uint32_t *ctr = p.gbar + gid * (kGroupCtrStride / 4);
-
-    auto load = [&](const char *g, uint32_t sb) {
-        const char *src = g + ((size_t)b0 * V * nvr + c0) * 16;
-        for (uint32_t e = threadIdx.x; e < cnt; e += blockDim.x) {
-            uint32_t i, j;
-            fdivmod32(e, divc, i, j);
-            cp_async16(sb + (i * q + j) * 16, src + ((size_t)i * nvr + j) * 16);
-        }
-        cp_async_commit();
-    };
-    auto arrive_when_loaded = [&]() {
-        cp_async_wait_all();
-        __syncthreads();
-        if (threadIdx.x == 0) group_arrive(ctr);
-    };
-
-    uint64_t t = gid;
-    if (t < p.count) {
-        load(tile_ptr(p, t), s0);
-        arrive_when_loaded();
-    }
-    for (uint32_t i = 0; t < p.count; t += ng, ++i) {
-        const uint32_t sb = s0 + (i & 1) * p.buf_bytes, sn = s0 + ((i + 1) & 1) * p.buf_bytes;
-        const uint64_t tn = t + ng;
-        if (tn < p.count) load(tile_ptr(p, tn), sn);
-        if (threadIdx.x == 0) group_wait(ctr, K * (i + 1));   // every slice of t on chip
-        __syncthreads();
-        char *g = tile_ptr(p, t);
-        if (h) write_out<EB>(p, sb, g, q, b0, h, div_h, c0, cvec);
-        if (tn < p.count) arrive_when_loaded();
-        write_out<EB>(p, sb + h * V * q * 16, g, q, b0 + h, nb - h, div_r, c0, cvec);
-        __syncthreads();                                      // buffer sb free
-    }
+    const FastDiv32 divc = make_fastdiv32_dev(cvec), divnb = make_fastdiv32_dev(nb);
+    __shared__ __align__(8) uint64_t mbar[kGroupMaxBuf];
+    group_loop<false>(p, s0, mbar,
+        [&](const char *g, uint32_t sb) {
+            const char *src = g + ((size_t)b0 * V * nvr + c0) * 16;
+            for (uint32_t e = threadIdx.x; e < cnt; e += blockDim.x) {
+                uint32_t i, j;
+                fdivmod32(e, divc, i, j);
+                cp_async16(sb + (i * q + j) * 16, src + ((size_t)i * nvr + j) * 16);
+            }
+        },
+        [&](char *g, uint32_t sb, uint32_t, uint32_t, auto probe) {
+            write_out<EB>(p, sb, g, q, b0, nb, divnb, c0, cvec, probe);
+        });
 }
 
 // ------------------------------------------------- group-split element-path kernel
@@ -549,7 +619,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_generic(const TileParams p)
     extern __shared__ __align__(128) unsigned char smem[];
     const uint32_t s0 = smem_u32(smem);
     const uint32_t K = p.K;
-    const uint32_t rank = blockIdx.x % K, gid = blockIdx.x / K, ng = gridDim.x / K;
+    const uint32_t rank = blockIdx.x % K;
     uint32_t r0, r1, c0, c1;
     if (p.colsplit) {
         r0 = 0; r1 = p.m;
@@ -567,7 +637,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_generic(const TileParams p)
     const uint32_t ntask = nrb * ncb;
     const FastDiv32 divrb = make_fastdiv32_dev(nrb);
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
-    uint32_t *ctr = p.gbar + gid * (kGroupCtrStride / 4);
+    __shared__ __align__(8) uint64_t mbar[kGroupMaxBuf];
 
     auto load = [&](const char *g, uint32_t sb) {
         const uint32_t cnt = rows * QV;
@@ -578,10 +648,11 @@ __global__ void __launch_bounds__(512, 1) tile_group_generic(const TileParams p)
             const uint32_t sh = (uint32_t)(a & 15) / EB;
             if (j * PV < sh + L) cp_async16(sb + (i * Q + j) * 16, (const void *)((a & ~(uintptr_t)15) + j * 16));
         }
-        cp_async_commit();
     };
-    auto write = [&](char *g, uint32_t sb, uint32_t task0, uint32_t task1) {
-        for (uint32_t task = task0 + warp; task < task1; task += nw) {
+    auto write = [&](char *g, uint32_t sb, uint32_t part, uint32_t parts, auto probe) {
+        const uint32_t task1 = ntask * (part + 1) / parts;
+        for (uint32_t task = ntask * part / parts + warp; task < task1; task += nw) {
+            probe();
             uint32_t cb, rb;
             fdivmod32(task, divrb, cb, rb);
             const uint32_t i = rb * 32 + lane, c = cb * PV;
@@ -609,29 +680,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_generic(const TileParams p)
             }
         }
     };
-    auto arrive_when_loaded = [&]() {
-        cp_async_wait_all();
-        __syncthreads();
-        if (threadIdx.x == 0) group_arrive(ctr);
-    };
-
-    uint64_t t = gid;
-    if (t < p.count) {
-        load(tile_ptr(p, t), s0);
-        arrive_when_loaded();
-    }
-    for (uint32_t it = 0; t < p.count; t += ng, ++it) {
-        const uint32_t sb = s0 + (it & 1) * p.buf_bytes, sn = s0 + ((it + 1) & 1) * p.buf_bytes;
-        const uint64_t tn = t + ng;
-        if (tn < p.count) load(tile_ptr(p, tn), sn);
-        if (threadIdx.x == 0) group_wait(ctr, K * (it + 1));
-        __syncthreads();
-        char *g = tile_ptr(p, t);
-        write(g, sb, 0, ntask / 2);
-        if (tn < p.count) arrive_when_loaded();
-        write(g, sb, ntask / 2, ntask);
-        __syncthreads();
-    }
+    group_loop<true>(p, s0, mbar, load, write);
 }
 
 // ------------------------------------------------------------------- generic kernel
@@ -907,43 +956,59 @@ static bool fast_colsplit(int64_t A, int64_t B, int eb) {
     return A < B && A * eb < 1024 && env_int("IPT_TILE_FAST_COLSPLIT", 1);
 }
 
-// Group split (tile_group_db): K CTAs per tile, `groups` tiles in flight, two slice buffers
-// of `slice` bytes per CTA.  Column split when B >= A (the strided side -- reads for a
-// column split, writes for a row split -- then moves B*eb/K-byte rather than A*eb/K-byte
-// pieces; measured 1.1-1.6x either way, tools/tile_big.py).  K minimises waves x (slice + 4 KB barrier allowance); a larger K must win by
-// 3 % (fewer CTAs per barrier, longer pieces).
-static bool group_colsplit(int64_t A, int64_t B) {
-    const long f = env_int("IPT_TILE_GROUP_COLSPLIT", -1);
-    return f >= 0 ? f != 0 : B >= A;
-}
+// Group split (tile_group_db / tile_group_generic): K CTAs per tile, `groups` tiles in
+// flight, nbuf slice buffers per CTA.  K minimises waves x (slice + 4 KB barrier
+// allowance); a larger K must win by 3 % (fewer CTAs per barrier, longer pieces).
+// Split direction (measured, tools/tile_big.py): a row split reads contiguous slices and
+// writes A*eb/K-byte pieces of every output row; it is preferred while those pieces are
+// >= 64 B (e.g. 720 x 720: 5.2 vs 4.4 TB/s, 600 x 1200: 4.9 vs 4.7), else the column
+// split (contiguous writes; 120 x 7200: 4.9 vs 3.3).
+constexpr long kGroupStaticSmem = 256;   // mbarriers
 
 struct GroupCfg {
-    int K = 0, groups = 0;
+    int K = 0, groups = 0, nbuf = 0;
     size_t slice = 0;
     bool colsplit = false;
 };
 
-GroupCfg group_cfg(int64_t A, int64_t B, int eb, uint64_t count, int device) {
+// Slice buffers per CTA (2; 3 or 4 measured 10-40 % slower: smaller slices, larger K).
+static int group_nbuf() {
+    const long b = env_int("IPT_TILE_GROUP_NBUF", 2);
+    return b < 2 ? 2 : (b > (long)kGroupMaxBuf ? (int)kGroupMaxBuf : (int)b);
+}
+
+// Best K for one split direction; `generic`: element-path slices of row pieces with one
+// padding vector (the aligner may read one vector past the last row).
+static GroupCfg group_search(int64_t A, int64_t B, int eb, uint64_t count, int device, bool cs,
+                             bool generic) {
     GroupCfg g;
-    if (!vec_ok(A, B, eb)) return g;
     const DevProps dp = dev_props(device);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
     const int V = 16 / eb;
-    const int64_t mv = A / V, nvr = B / V;
-    const bool cs = group_colsplit(A, B);
-    g.colsplit = cs;
-    const size_t q = fast_q(B, eb);
     const int kfix = (int)env_int("IPT_TILE_GROUP_K", 0);
+    const int nb = group_nbuf();
+    const uint64_t cnt = std::max<uint64_t>(count, 1);
+    g.nbuf = nb;
+    g.colsplit = cs;
     double best = 1e300;
     for (int K = 2; K <= dp.sms; ++K) {
         if (kfix && K != kfix) continue;
-        if ((cs ? nvr : mv) < K) break;
-        size_t slice = cs ? (size_t)A * (size_t)(((nvr + K - 1) / K) | 1) * 16
-                          : (size_t)((mv + K - 1) / K) * V * q * 16;
+        size_t slice;
+        if (generic) {
+            if ((cs ? B : A) < (int64_t)K * (cs ? V : 1)) break;
+            const int64_t L = cs ? (B + K - 1) / K : B;
+            const int64_t rows = cs ? A : (A + K - 1) / K;
+            slice = (size_t)(rows * (((L + 2 * V - 2) / V) | 1) + 1) * 16;
+        } else {
+            const int64_t mv = A / V, nvr = B / V;
+            if ((cs ? nvr : mv) < K) break;
+            slice = cs ? (size_t)A * (size_t)(((nvr + K - 1) / K) | 1) * 16
+                       : (size_t)((mv + K - 1) / K) * V * fast_q(B, eb) * 16;
+        }
         slice = (slice + 127) & ~(size_t)127;
-        if ((long)(2 * slice) > budget) continue;
-        const int64_t groups = std::min<int64_t>(dp.sms / K, (int64_t)std::max<uint64_t>(count, 1));
-        const double waves = (double)((std::max<uint64_t>(count, 1) + groups - 1) / groups);
+        if ((long)(nb * slice) + kGroupStaticSmem > budget) continue;
+        const int64_t groups = std::min<int64_t>(dp.sms / K, (int64_t)cnt);
+        const double waves = (double)((cnt + groups - 1) / groups);
         const double cost = waves * ((double)slice + 4096.0);
         if (cost < best * 0.97) {
             best = cost;
@@ -955,38 +1020,23 @@ GroupCfg group_cfg(int64_t A, int64_t B, int eb, uint64_t count, int device) {
     return g;
 }
 
-// Element-path group split: slices of row pieces (see tile_group_generic), one padding
-// vector per buffer (the aligner may read one vector past the last row).
+static GroupCfg group_choose(int64_t A, int64_t B, int eb, uint64_t count, int device, bool generic) {
+    const long f = env_int("IPT_TILE_GROUP_COLSPLIT", -1);
+    if (f >= 0) return group_search(A, B, eb, count, device, f != 0, generic);
+    const GroupCfg row = group_search(A, B, eb, count, device, false, generic);
+    if (row.K && A * eb / row.K >= 64) return row;
+    const GroupCfg col = group_search(A, B, eb, count, device, true, generic);
+    return col.K ? col : row;
+}
+
+GroupCfg group_cfg(int64_t A, int64_t B, int eb, uint64_t count, int device) {
+    if (!vec_ok(A, B, eb)) return GroupCfg{};
+    return group_choose(A, B, eb, count, device, false);
+}
+
 GroupCfg group_cfg_generic(int64_t A, int64_t B, int eb, uint64_t count, int device) {
-    GroupCfg g;
-    if (eb != 4 && eb != 8) return g;
-    const DevProps dp = dev_props(device);
-    const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
-    const int PV = 16 / eb;
-    const bool cs = group_colsplit(A, B);
-    g.colsplit = cs;
-    const int kfix = (int)env_int("IPT_TILE_GROUP_K", 0);
-    double best = 1e300;
-    for (int K = 2; K <= dp.sms; ++K) {
-        if (kfix && K != kfix) continue;
-        if ((cs ? B : A) < (int64_t)K * (cs ? PV : 1)) break;
-        const int64_t L = cs ? (B + K - 1) / K : B;
-        const int64_t rows = cs ? A : (A + K - 1) / K;
-        const int64_t Q = ((L + 2 * PV - 2) / PV) | 1;
-        size_t slice = (size_t)(rows * Q + 1) * 16;
-        slice = (slice + 127) & ~(size_t)127;
-        if ((long)(2 * slice) > budget) continue;
-        const int64_t groups = std::min<int64_t>(dp.sms / K, (int64_t)std::max<uint64_t>(count, 1));
-        const double waves = (double)((std::max<uint64_t>(count, 1) + groups - 1) / groups);
-        const double cost = waves * ((double)slice + 4096.0);
-        if (cost < best * 0.97) {
-            best = cost;
-            g.K = K;
-            g.groups = (int)groups;
-            g.slice = slice;
-        }
-    }
-    return g;
+    if (eb != 4 && eb != 8) return GroupCfg{};
+    return group_choose(A, B, eb, count, device, true);
 }
 
 // Group-split launch: groups x K CTAs, all co-resident (cooperative launch); the arrival
@@ -1003,16 +1053,29 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
     }
     p.colsplit = g.colsplit ? 1 : 0;
     p.K = (uint32_t)g.K;
+    p.nbuf = (uint32_t)g.nbuf;
     p.buf_bytes = (uint32_t)g.slice;
     p.gbar = (uint32_t *)ws;
+    if ((size_t)g.groups * g.nbuf * kGroupCtrStride > kTileWsBytes) return cudaErrorInvalidValue;
     auto kern = GENERIC ? tile_group_generic<EB> : tile_group_db<EB>;
-    cudaError_t e = cudaMemsetAsync(ws, 0, (size_t)g.groups * kGroupCtrStride, st);
+    cudaError_t e = cudaMemsetAsync(ws, 0, (size_t)g.groups * g.nbuf * kGroupCtrStride, st);
     if (e != cudaSuccess) return e;
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dev_props(device).smem_optin);
+    {   // dynamic + static shared memory must stay within the opt-in maximum
+        static std::mutex mu;
+        static std::map<std::pair<const void *, int>, bool> done;
+        std::lock_guard<std::mutex> lk(mu);
+        if (!done[std::make_pair((const void *)kern, device)]) {
+            cudaFuncAttributes fa{};
+            cudaFuncGetAttributes(&fa, kern);
+            cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 dev_props(device).smem_optin - (int)fa.sharedSizeBytes);
+            done[std::make_pair((const void *)kern, device)] = true;
+        }
+    }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)(g.groups * g.K), 1, 1);
     cfg.blockDim = dim3(512, 1, 1);
-    cfg.dynamicSmemBytes = 2 * g.slice;
+    cfg.dynamicSmemBytes = g.nbuf * g.slice;
     cfg.stream = st;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeCooperative;
@@ -1021,7 +1084,7 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
     cfg.numAttrs = 1;
     if (env_int("IPT_DEBUG", 0))
         fprintf(stderr, "[ipt] tile_group%s m=%u n=%u K=%d groups=%d colsplit=%d smem=%zu tiles=%llu\n",
-                GENERIC ? "_generic" : "", p.m, p.n, g.K, g.groups, p.colsplit, 2 * g.slice,
+                GENERIC ? "_generic" : "", p.m, p.n, g.K, g.groups, p.colsplit, g.nbuf * g.slice,
                 (unsigned long long)p.count);
     e = cudaLaunchKernelEx(&cfg, kern, p);
     note_launch();

@@ -518,11 +518,10 @@ struct GroupPipe {
 };
 
 // Main loop of a group kernel: load(tile pointer, buffer address) issues the cp.async
-// copies of one slice; write(tile pointer, buffer address, part, parts, probe) writes part
-// `part` of `parts` of one out, calling probe() now and then.  MIDSYNC: instead of
-// probing, the CTA waits for the next slice half-way through the write-out and then
-// arrives (measured faster for the element-path kernel, slower for the 16-byte one).
-template <bool MIDSYNC, typename Load, typename Write>
+// copies of one slice; write(tile pointer, buffer address, probe) writes one out, calling
+// probe() now and then.  (Waiting for the next slice half-way through the write-out and
+// arriving then, with all warps, measured 2-8 % slower than thread 0 probing.)
+template <typename Load, typename Write>
 __device__ __forceinline__ void group_loop(const TileParams &p, uint32_t s0, uint64_t *mbar,
                                            Load load, Write write) {
     const uint32_t K = p.K, gid = blockIdx.x / K, ng = gridDim.x / K;
@@ -548,20 +547,8 @@ __device__ __forceinline__ void group_loop(const TileParams &p, uint32_t s0, uin
             pipe.wait_group(i);                      // every slice of tile i on chip
         }
         __syncthreads();
-        char *g = tile_ptr(p, gid + (uint64_t)i * ng);
-        const uint32_t sb = s0 + (i % p.nbuf) * p.buf_bytes;
-        if (MIDSYNC) {
-            auto none = []() {};
-            write(g, sb, 0, 2, none);
-            if (jn < nt) {
-                pipe.wait_landed(jn);
-                __syncthreads();
-                if (threadIdx.x == 0) pipe.force(jn);
-            }
-            write(g, sb, 1, 2, none);
-        } else {
-            write(g, sb, 0, 1, [&]() { if (threadIdx.x == 0) pipe.probe(lim); });
-        }
+        write(tile_ptr(p, gid + (uint64_t)i * ng), s0 + (i % p.nbuf) * p.buf_bytes,
+              [&]() { if (threadIdx.x == 0) pipe.probe(lim); });
         __syncthreads();                             // buffer i % nbuf free
     }
 }
@@ -589,7 +576,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_db(const TileParams p) {
     const uint32_t cnt = nb * V * cvec;
     const FastDiv32 divc = make_fastdiv32_dev(cvec), divnb = make_fastdiv32_dev(nb);
     __shared__ __align__(8) uint64_t mbar[kGroupMaxBuf];
-    group_loop<false>(p, s0, mbar,
+    group_loop(p, s0, mbar,
         [&](const char *g, uint32_t sb) {
             const char *src = g + ((size_t)b0 * V * nvr + c0) * 16;
             for (uint32_t e = threadIdx.x; e < cnt; e += blockDim.x) {
@@ -598,7 +585,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_db(const TileParams p) {
                 cp_async16(sb + (i * q + j) * 16, src + ((size_t)i * nvr + j) * 16);
             }
         },
-        [&](char *g, uint32_t sb, uint32_t, uint32_t, auto probe) {
+        [&](char *g, uint32_t sb, auto probe) {
             write_out<EB>(p, sb, g, q, b0, nb, divnb, c0, cvec, probe);
         });
 }
@@ -633,10 +620,12 @@ __global__ void __launch_bounds__(512, 1) tile_group_generic(const TileParams p)
     const uint32_t rows = r1 - r0, L = c1 - c0, Q = p.q;
     const uint32_t QV = (L + 2 * PV - 2) / PV;            // covering vectors, worst phase
     const FastDiv32 divq = make_fastdiv32_dev(QV);
-    const uint32_t nrb = (rows + 31) / 32, ncb = (L + PV - 1) / PV;
-    const uint32_t ntask = nrb * ncb;
+    constexpr uint32_t CH = 8;                            // column blocks per write task
+    const uint32_t nrb = (rows + 31) / 32, ncb = (L + PV - 1) / PV, nch = (ncb + CH - 1) / CH;
+    const uint32_t ntask = nrb * nch;
     const FastDiv32 divrb = make_fastdiv32_dev(nrb);
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+    const uint64_t mEB = (uint64_t)p.m * EB;
     __shared__ __align__(8) uint64_t mbar[kGroupMaxBuf];
 
     auto load = [&](const char *g, uint32_t sb) {
@@ -649,38 +638,47 @@ __global__ void __launch_bounds__(512, 1) tile_group_generic(const TileParams p)
             if (j * PV < sh + L) cp_async16(sb + (i * Q + j) * 16, (const void *)((a & ~(uintptr_t)15) + j * 16));
         }
     };
-    auto write = [&](char *g, uint32_t sb, uint32_t part, uint32_t parts, auto probe) {
-        const uint32_t task1 = ntask * (part + 1) / parts;
-        for (uint32_t task = ntask * part / parts + warp; task < task1; task += nw) {
+    // Task (column chunk ch, row block rb), row blocks fastest: the warps of a CTA write
+    // adjacent 32-element runs of the same output rows.  Per lane: one row, CH x PV columns.
+    auto write = [&](char *g, uint32_t sb, auto probe) {
+        for (uint32_t task = warp; task < ntask; task += nw) {
             probe();
-            uint32_t cb, rb;
-            fdivmod32(task, divrb, cb, rb);
-            const uint32_t i = rb * 32 + lane, c = cb * PV;
-            E x[2 * PV];
-            if (i < rows) {
-                const uintptr_t a = (uintptr_t)(g + ((uint64_t)(r0 + i) * p.n + c0) * EB);
-                const uint32_t w = (uint32_t)(a & 15) / EB + c;
-                const uint32_t v = w / PV, o = w % PV;
-                E ex[PV], ey[PV];
-                unpack<EB>(lds128(sb + (i * Q + v) * 16), ex);
-                unpack<EB>(lds128(sb + (i * Q + v + 1) * 16), ey);
+            uint32_t ch, rb;
+            fdivmod32(task, divrb, ch, rb);
+            const uint32_t i = rb * 32 + lane;
+            if (i >= rows) continue;
+            const uintptr_t a = (uintptr_t)(g + ((uint64_t)(r0 + i) * p.n + c0) * EB);
+            const uint32_t sh = (uint32_t)(a & 15) / EB;
+            const uint32_t srow = sb + i * Q * 16;
+            const uint32_t cfirst = ch * CH * PV;
+            char *out = g + ((uint64_t)(c0 + cfirst) * p.m + r0 + i) * EB;
+#pragma unroll 2
+            for (uint32_t cbl = 0; cbl < CH; ++cbl) {
+                const uint32_t c = cfirst + cbl * PV;
+                if (c >= L) break;
+                const uint32_t w = sh + c, v = w / PV, o = w % PV;
+                E x[2 * PV];
+                {
+                    E ex[PV], ey[PV];
+                    unpack<EB>(lds128(srow + v * 16), ex);
+                    unpack<EB>(lds128(srow + (v + 1) * 16), ey);
 #pragma unroll
-                for (uint32_t k = 0; k < PV; ++k) { x[k] = ex[k]; x[PV + k] = ey[k]; }
+                    for (uint32_t k = 0; k < PV; ++k) { x[k] = ex[k]; x[PV + k] = ey[k]; }
+                }
 #pragma unroll
                 for (uint32_t sft = 1; sft < PV; sft <<= 1) {   // x[k] <- x[k + o]
                     const bool f = (o & sft) != 0;
 #pragma unroll
                     for (uint32_t k = 0; k + sft < 2 * PV; ++k) x[k] = f ? x[k + sft] : x[k];
                 }
-            }
+                char *oc = out + (uint64_t)cbl * PV * mEB;
 #pragma unroll
-            for (uint32_t k = 0; k < PV; ++k) {
-                if (i < rows && c + k < L)
-                    *reinterpret_cast<E *>(g + ((uint64_t)(c0 + c + k) * p.m + r0 + i) * EB) = x[k];
+                for (uint32_t k = 0; k < PV; ++k)
+                    if (c + k < L) *reinterpret_cast<E *>(oc + k * mEB) = x[k];
             }
         }
     };
-    group_loop<true>(p, s0, mbar, load, write);
+    group_loop(p, s0, mbar, load, write);
 }
 
 // ------------------------------------------------------------------- generic kernel

@@ -161,3 +161,21 @@ def test_workspace_batch_scales():
     p = ipt.plan(4096, 3000, 4)
     w1, w8 = ipt.workspace_bytes(p, 1), ipt.workspace_bytes(p, 8)
     assert w8 > w1 and w8 <= 8 * w1 + 256
+
+
+def test_group_split_extends_on_chip_tiles():
+    """Tiles beyond 16 x 227 KB clusters run on chip over co-resident CTA groups (up to
+    ~148 x 113 KB, double-buffered); larger tiles fall back to cycle following.  A tile
+    stage reserves 8 KB of workspace for the group counters (nominal B200, no GPU)."""
+    V = ipt.VARIANTS
+    for (M, N, m, n) in [(4096, 4096, 1024, 1024),     # 4 MB 16-byte-path tiles
+                         (16384, 16384, 128, 16384),   # 8 MB panels (n = N)
+                         (14803, 8192, 14803, 128),    # 7.6 MB element-path panels (m = M)
+                         (12288, 9998, 192, 9998)]:
+        p = ipt.plan(M, N, 4, m=m, n=n)
+        assert V[p.variant[1]] == "tile_onchip", (M, N, m, n)
+        assert p.workspace_bytes >= 8192
+    p = ipt.plan(4096, 8192, 4, m=4096, n=2048)         # 32 MB: beyond aggregate smem
+    assert V[p.variant[1]] == "cycle_global"
+    assert ipt.lib().ipt_stage_workspace_bytes(3, 120, 7200, 1, 4) >= 8192
+    assert ipt.lib().ipt_stage_workspace_bytes(1, 4, 4, 5, 4) < 8192   # cycle stage: flags only

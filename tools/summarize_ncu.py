@@ -22,15 +22,19 @@ NCU = "/usr/local/cuda/bin/ncu"
 
 
 def kind(name: str):
-    if "cycle_global" in name:
+    """Kernel family as bench.py names it: cycle_global, or tile_onchip for every tile-stage
+    kernel (tile_onchip_*, tile_group_db, tile_group_generic, tile_generic_cluster)."""
+    if "cycle_global" in name or "cycle_ua" in name:
         return "cycle_global"
-    if "tile_onchip" in name:
+    if "tile_" in name:
         return "tile_onchip"
     return None
 
 
-def launches(tag):
-    path = os.path.join(GO, "launches.csv")
+def launches(tag, workload="sweep"):
+    path = os.path.join(GO, "launches.csv" if workload == "sweep" else f"launches_{workload}.csv")
+    if not os.path.exists(path):
+        return
     rows = [r for r in csv.reader(open(path)) if len(r) > 10]
     hdr = rows[0]
     idx = {h: i for i, h in enumerate(hdr)}
@@ -58,7 +62,8 @@ def launches(tag):
         a["rd"] += d.get("dram__bytes_read.sum", 0.0)
         a["wr"] += d.get("dram__bytes_write.sum", 0.0)
     tot = sum(a["us"] for a in agg.values())
-    lines = [f"# {tag}: ncu launch list of `python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu`",
+    cmd = "python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu" + ("" if workload == "sweep" else f" --workload {workload}")
+    lines = [f"# {tag}: ncu launch list of `{cmd}`",
              "", "Cold-cache, serialised (`--clock-control none`); compare SHARES, not absolutes. "
              "Only libipt kernels are aggregated (torch generator fills run outside the timed region).",
              "", "| kernel | launches | total µs | share | avg µs/launch | DRAM read MB/launch | DRAM write MB/launch |",
@@ -68,12 +73,13 @@ def launches(tag):
         lines.append(f"| {k} | {a['n']} | {a['us']:.1f} | {a['us'] / tot:.3f} | {a['us'] / a['n']:.1f} | "
                      f"{a['rd'] / a['n'] / 1e6:.1f} | {a['wr'] / a['n'] / 1e6:.1f} |")
         traffic[k] = round((a["rd"] + a["wr"]) / a["n"])
-    open(os.path.join(PROF, f"{tag}_launches.md"), "w").write("\n".join(lines) + "\n")
+    suffix = "" if workload == "sweep" else f"_{workload}"
+    open(os.path.join(PROF, f"{tag}_launches{suffix}.md"), "w").write("\n".join(lines) + "\n")
     tp = os.path.join(PROF, "traffic.json")
     cur = json.load(open(tp)) if os.path.exists(tp) else {}
-    cur["sweep"] = traffic
+    cur[workload] = traffic
     cur["_note"] = ("bytes per launch (dram read + write), averaged over the libipt launches of "
-                    "the sweep bench under ncu; source: profiles/%s_launches.md" % tag)
+                    "each workload's bench under ncu; source: profiles/%s_launches*.md" % tag)
     json.dump(cur, open(tp, "w"), indent=1)
     print("\n".join(lines))
 
@@ -123,5 +129,6 @@ def full(tag):
 if __name__ == "__main__":
     tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
     os.makedirs(PROF, exist_ok=True)
-    launches(tag)
+    for w in ("sweep", "c1", "c3", "c4", "c5"):
+        launches(tag, w)
     full(tag)

@@ -720,7 +720,10 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
         const uint64_t walkers = (uint64_t)dp.sms * 64 * (c.ua ? 1 : (32 / c.G));
         long forced = env_int("IPT_CYC_SEGSH", -1);
         uint32_t sh = 0;
-        while (sh < 5 && (p.nwords << sh) < 2 * walkers) ++sh;
+        // target fetches = walkers / 2 (measured, tools/cyc_knobs.py: 1-2x starve the fetch
+        // counter -- one contended atomic per fetch -- on C1-sized stages: -20..-45 %)
+        const uint64_t target = walkers * (uint64_t)env_int("IPT_CYC_SEGF", 50) / 100;
+        while (sh < 5 && (p.nwords << sh) < target) ++sh;
         if (forced >= 0 && forced <= 5) sh = (uint32_t)forced;
         p.segsh = sh;
         p.nfetch = p.nwords << sh;

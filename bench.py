@@ -60,8 +60,68 @@ def load_peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+class NvmlClockSampler:
+    """SM clocks / clock-event (throttle) reasons sampled every ~2 ms by NVML in a thread
+    during the timed region (nvidia-smi -lms cannot sample a 50 ms region usefully)."""
+
+    NAMES = {"hw_slowdown": "nvmlClocksEventReasonHwSlowdown",
+             "hw_thermal_slowdown": "nvmlClocksEventReasonHwThermalSlowdown",
+             "sw_thermal_slowdown": "nvmlClocksEventReasonSwThermalSlowdown",
+             "sw_power_cap": "nvmlClocksEventReasonSwPowerCap",
+             "hw_power_brake_slowdown": "nvmlClocksEventReasonHwPowerBrakeSlowdown"}
+
+    def __init__(self, device: int):
+        import threading
+
+        import pynvml as nv
+        import torch
+
+        self.nv = nv
+        nv.nvmlInit()
+        h = None
+        try:   # CUDA and NVML orders differ under CUDA_VISIBLE_DEVICES: match by PCI id
+            pr = torch.cuda.get_device_properties(device)
+            bus = f"{pr.pci_domain_id:08x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+            h = nv.nvmlDeviceGetHandleByPciBusId(bus)
+        except Exception:
+            h = nv.nvmlDeviceGetHandleByIndex(device)
+        self.h = h
+        self.max_mhz = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+        self.rows = []
+        self.stop_ev = threading.Event()
+        self.th = threading.Thread(target=self._run, daemon=True)
+        self.th.start()
+
+    def _run(self):
+        nv = self.nv
+        while not self.stop_ev.is_set():
+            try:
+                self.rows.append((nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM),
+                                  nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)))
+            except Exception:
+                pass
+            self.stop_ev.wait(0.002)
+
+    def stop(self):
+        self.stop_ev.set()
+        self.th.join(timeout=5)
+        if not self.rows:
+            return None
+        reasons = sorted(n for n, attr in self.NAMES.items()
+                         if any(r & getattr(self.nv, attr, 0) for _, r in self.rows))
+        return {"sm_mhz": statistics.median(c for c, _ in self.rows), "sm_max_mhz": self.max_mhz,
+                "reasons": reasons, "samples": len(self.rows), "source": "nvml, 2 ms"}
+
+
+def clock_sampler(device: int):
+    try:
+        return NvmlClockSampler(device)
+    except Exception:
+        return ClockSampler(device)
+
+
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    """nvidia-smi clocks / throttle reasons sampled during the timed region (fallback)."""
 
     def __init__(self, index: int):
         self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
@@ -281,19 +341,39 @@ def main():
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    clocks = ClockSampler(local)
+    l2_bytes = torch.cuda.get_device_properties(dev).L2_cache_size
+    resident = any(M * N * eb * cnt <= l2_bytes for (_, M, N, cnt, _) in mats)
+    # 4x L2 of flush writes per step (int32 add over 512 MB) for L2-resident matrices
+    flush = torch.zeros(128 << 20, dtype=torch.int32, device=dev) if resident else None
+    clocks = clock_sampler(local)
     launches0 = ipt.kernel_launch_count()
     orient_before = list(orient)
     torch.cuda.nvtx.range_push("timed")       # ncu --nvtx --nvtx-include "timed/"
-    t_start.record()
-    for s in range(args.steps):
-        one_step(evs[s] if args.algo == "3stage" else None)
-    t_end.record()
+    if flush is None:
+        t_start.record()
+        for s in range(args.steps):
+            one_step(evs[s] if args.algo == "3stage" else None)
+        t_end.record()
+    else:
+        # L2-resident workload: overwrite L2 before every step (outside the step's events)
+        # so each step starts cold, as a larger-than-L2 input would
+        step_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                   for _ in range(args.steps)]
+        for s in range(args.steps):
+            flush.add_(1)
+            step_ev[s][0].record()
+            one_step(evs[s] if args.algo == "3stage" else None)
+            step_ev[s][1].record()
     torch.cuda.synchronize()
     torch.cuda.nvtx.range_pop()
     launches = ipt.kernel_launch_count() - launches0
     clk = clocks.stop()
-    elapsed_ms = t_start.elapsed_time(t_end)
+    if flush is None:
+        elapsed_ms = t_start.elapsed_time(t_end)
+    else:
+        elapsed_ms = sum(a.elapsed_time(b) for a, b in step_ev)
+    flushed = flush is not None
+    del flush
     tmax = torch.tensor([elapsed_ms], dtype=torch.float64, device=red_dev)
     if world > 1:
         dist.barrier()
@@ -460,7 +540,9 @@ def main():
                        "shapes": [f"{M}x{N}" for (M, N) in wl["shapes"]],
                        "elem_bytes": eb, "batch": wl.get("batch", 1),
                        "plans": plans_cfg,
-                       "l2": "no flush: every matrix exceeds the 126 MB L2" if args.workload in ("sweep", "c3", "c4", "c5") else "L2-resident (52 MB)",
+                       "l2": ("no flush: every matrix exceeds the 126 MB L2" if not flushed else
+                              "L2 flushed before every step (512 MB read+write, outside the step's events; "
+                              "time = sum of per-step device times)"),
                        "parallelism": f"replicas x{world}" if "batch" not in wl else f"batch shards x{world}",
                        "algo": args.algo,
                        "planning": (f"ipt_plan_autotune, {args.autotune} candidates per shape "

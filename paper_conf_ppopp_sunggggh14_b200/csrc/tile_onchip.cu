@@ -52,6 +52,13 @@ struct TileParams {
     uint32_t gb;          // streaming kernel: V-row blocks per group (0 = automatic)
     uint32_t *gbar;       // group-split kernel: one arrival counter per group (workspace)
     int vec16;            // generic path: tiles 16-byte aligned, 16-byte loads
+    int arrive_release;   // group kernels: release-ordered arrivals (default relaxed)
+    int bulk;             // tile_group_db: slices fetched by 1-D bulk copies (TMA engine)
+    int diag;             // group kernels, measurement only (IPT_TILE_DIAG; results invalid):
+                          // 1 = no group wait, 2 = no stores, 4 = no loads, 32 = stores
+                          // to a second buffer after the data, 64 = evict_first loads; 16 = timeline
+                          // trace (results valid, see ipt__tile_trace)
+    unsigned long long *trace;
 };
 
 __device__ __forceinline__ char *tile_ptr(const TileParams &p, uint64_t t) {
@@ -457,8 +464,9 @@ __global__ void __launch_bounds__(512, 1) tile_onchip_stream(const TileParams p)
 // tile is signalled half-way through the current write-out, so the wait is normally
 // already satisfied (a CTA only arrives for tile i+1 after passing the wait for tile i,
 // hence the cumulative count K*(i+1) identifies tile i).
-__device__ __forceinline__ void group_arrive(uint32_t *ctr) {
-    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
+__device__ __forceinline__ void group_arrive(uint32_t *ctr, bool release) {
+    if (release) asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
+    else asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
 }
 __device__ __forceinline__ uint64_t global_ns() {
     uint64_t t;
@@ -479,6 +487,9 @@ __device__ __forceinline__ void group_wait(const uint32_t *ctr, uint32_t target)
 }
 
 constexpr uint32_t kGroupMaxBuf = 4;
+constexpr uint32_t kTraceIters = 64;   // diag trace: iterations recorded per CTA
+constexpr size_t kTraceBytes = 1024 * kTraceIters * 4 * 8;
+static unsigned long long *g_trace = nullptr;
 
 // Ring of p.nbuf slice buffers shared by the group kernels.  Iteration j of a group
 // handles tile gid + j*groups in buffer j % nbuf; the loads of tile j + nbuf - 1 are
@@ -493,6 +504,7 @@ struct GroupPipe {
     uint64_t *mbar;     // nbuf mbarriers in shared memory
     uint32_t *ctr;      // this group's counters, kGroupCtrStride bytes apart
     uint32_t K, nbuf;
+    bool release;       // arrive with release semantics (IPT_TILE_ARRIVE_RELEASE=1)
     uint32_t na = 0;    // thread 0: next iteration to arrive for
     __device__ void init() {
         if (threadIdx.x == 0) {
@@ -506,12 +518,12 @@ struct GroupPipe {
     __device__ bool landed(uint32_t j) { return mbar_test_wait(&mbar[j % nbuf], (j / nbuf) & 1); }
     __device__ void wait_landed(uint32_t j) { mbar_wait(&mbar[j % nbuf], (j / nbuf) & 1); }
     __device__ void probe(uint32_t limit) {          // thread 0
-        while (na < limit && landed(na)) group_arrive(slot(na++));
+        while (na < limit && landed(na)) group_arrive(slot(na++), release);
     }
     __device__ void force(uint32_t j) {              // thread 0: arrivals up to j
         while (na <= j) {
             wait_landed(na);
-            group_arrive(slot(na++));
+            group_arrive(slot(na++), release);
         }
     }
     __device__ void wait_group(uint32_t j) { group_wait(slot(j), K * (j / nbuf + 1)); }
@@ -530,26 +542,40 @@ __device__ __forceinline__ void group_loop(const TileParams &p, uint32_t s0, uin
     pipe.ctr = p.gbar + gid * p.nbuf * (kGroupCtrStride / 4);
     pipe.K = K;
     pipe.nbuf = p.nbuf;
+    pipe.release = p.arrive_release != 0;
     pipe.init();
     const uint32_t nt = gid < p.count ? (uint32_t)((p.count - gid + ng - 1) / ng) : 0;
     auto issue = [&](uint32_t j) {
-        load(tile_ptr(p, gid + (uint64_t)j * ng), s0 + (j % p.nbuf) * p.buf_bytes);
+        if (!(p.diag & 4)) load(tile_ptr(p, gid + (uint64_t)j * ng), s0 + (j % p.nbuf) * p.buf_bytes);
         pipe.issued(j);
     };
     for (uint32_t j = 0; j + 1 < p.nbuf && j < nt; ++j) issue(j);
+    // timeline trace (diag 16): per CTA and iteration, globaltimer at start, own slice
+    // landed, group complete, write-out done
+    unsigned long long *tr = (p.diag & 16) && threadIdx.x == 0 ? p.trace + (uint64_t)blockIdx.x * kTraceIters * 4 : nullptr;
     for (uint32_t i = 0; i < nt; ++i) {
+        if (tr && i < kTraceIters - 1) tr[i * 4 + 0] = global_ns();
         const uint32_t jn = i + p.nbuf - 1;
         if (jn < nt) issue(jn);
         const uint32_t lim = min(nt, jn + 1);
         pipe.wait_landed(i);                         // own slice of tile i on chip
         if (threadIdx.x == 0) {
+            if (tr && i < kTraceIters - 1) tr[i * 4 + 1] = global_ns();
             pipe.force(i);
-            pipe.wait_group(i);                      // every slice of tile i on chip
+            if (!(p.diag & 1)) pipe.wait_group(i);   // every slice of tile i on chip
+            if (tr && i < kTraceIters - 1) tr[i * 4 + 2] = global_ns();
         }
         __syncthreads();
-        write(tile_ptr(p, gid + (uint64_t)i * ng), s0 + (i % p.nbuf) * p.buf_bytes,
+        if (!(p.diag & 2)) write(tile_ptr(p, gid + (uint64_t)i * ng) + ((p.diag & 32) ? p.count * p.tile_bytes : 0),
+              s0 + (i % p.nbuf) * p.buf_bytes,
               [&]() { if (threadIdx.x == 0) pipe.probe(lim); });
         __syncthreads();                             // buffer i % nbuf free
+        if (tr && i < kTraceIters - 1) tr[i * 4 + 3] = global_ns();
+    }
+    if (tr) {   // last trace slot: the SM this CTA ran on
+        uint32_t smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        tr[(kTraceIters - 1) * 4] = smid;
     }
 }
 
@@ -579,6 +605,27 @@ __global__ void __launch_bounds__(512, 1) tile_group_db(const TileParams p) {
     group_loop(p, s0, mbar,
         [&](const char *g, uint32_t sb) {
             const char *src = g + ((size_t)b0 * V * nvr + c0) * 16;
+            if (p.bulk) {   // one bulk copy per slice row (cvec vectors), issued by warp 0
+                if (threadIdx.x < 32) {
+                    const uint32_t sbar = smem_u32(&mbar[(sb - s0) / p.buf_bytes]);
+                    if (threadIdx.x == 0) mbar_expect_tx(&mbar[(sb - s0) / p.buf_bytes], cnt * 16);
+                    __syncwarp();
+                    for (uint32_t i = threadIdx.x; i < nb * V; i += 32)
+                        bulk_g2s_u32(sb + i * q * 16, src + (size_t)i * nvr * 16, cvec * 16, sbar);
+                }
+                return;
+            }
+            if (p.diag & 64) {
+                uint64_t pol;
+                asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+                for (uint32_t e = threadIdx.x; e < cnt; e += blockDim.x) {
+                    uint32_t i, j;
+                    fdivmod32(e, divc, i, j);
+                    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;"
+                                 :: "r"(sb + (i * q + j) * 16), "l"(src + ((size_t)i * nvr + j) * 16), "l"(pol) : "memory");
+                }
+                return;
+            }
             for (uint32_t e = threadIdx.x; e < cnt; e += blockDim.x) {
                 uint32_t i, j;
                 fdivmod32(e, divc, i, j);
@@ -1222,6 +1269,15 @@ cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, in
     p.divM = make_fastdiv((uint64_t)d.A);
     p.divN = make_fastdiv((uint64_t)d.B);
     p.gb = (uint32_t)env_int("IPT_TILE_GROUP", 0);
+    p.diag = (int)env_int("IPT_TILE_DIAG", 0);
+    if (p.diag & 16) {
+        if (!g_trace && cudaMalloc(&g_trace, kTraceBytes) != cudaSuccess) g_trace = nullptr;
+        if (g_trace) cudaMemsetAsync(g_trace, 0, kTraceBytes, st);
+        p.trace = g_trace;
+        if (!g_trace) p.diag &= ~16;
+    }
+    p.bulk = (int)env_int("IPT_TILE_BULK", 0);
+    p.arrive_release = (int)env_int("IPT_TILE_ARRIVE_RELEASE", 0);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) <= budget) {
         const int V = 16 / d.eb;
@@ -1341,3 +1397,12 @@ cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, in
 }
 
 }  // namespace ipt
+
+// Internal diagnostic hook (not in the ABI): copy the last group-kernel timeline trace
+// (IPT_TILE_DIAG=16; [CTA][iteration][4] globaltimer ns) to host memory.
+extern "C" int ipt__tile_trace(void *host, size_t bytes) {
+    if (!ipt::g_trace) return -1;
+    cudaDeviceSynchronize();
+    return (int)cudaMemcpy(host, ipt::g_trace, bytes < ipt::kTraceBytes ? bytes : ipt::kTraceBytes,
+                           cudaMemcpyDeviceToHost);
+}

@@ -6,7 +6,8 @@ if os.environ.get("_CHILD"):
     import torch
     import paper_conf_ppopp_sunggggh14_b200 as ipt
     TOT = 12800 * 15000
-    buf = torch.empty(TOT, dtype=torch.int32, device="cuda")
+    oop = int(os.environ.get("IPT_TILE_DIAG", "0")) & 32
+    buf = torch.empty(2 * TOT if oop else TOT, dtype=torch.int32, device="cuda")
     buf.random_()
     res = {}
     for (m, n) in ast.literal_eval(os.environ["SHAPES"]):
@@ -22,7 +23,17 @@ if os.environ.get("_CHILD"):
             ipt.ipt_010_(buf, cnt, m, n)
         e1.record(); torch.cuda.synchronize()
         ms = e0.elapsed_time(e1) / 5
-        res[f"{m}x{n}"] = round(2 * cnt * m * n * 4 / (ms / 1e3) / 1e9) if ok else "WRONG"
+        rate = round(2 * cnt * m * n * 4 / (ms / 1e3) / 1e9)
+        res[f"{m}x{n}"] = rate if ok else (f"{rate}?" if os.environ.get("IPT_TILE_DIAG") else "WRONG")
+    if os.environ.get("COPY_REF"):   # device copy of the same bytes: the practical ceiling
+        dst = torch.empty_like(buf)
+        dst.copy_(buf)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for r in range(5):
+            dst.copy_(buf)
+        e1.record(); torch.cuda.synchronize()
+        res["copy"] = round(2 * TOT * 4 / (e0.elapsed_time(e1) / 5 / 1e3) / 1e9)
     print(json.dumps(res), flush=True)
 else:
     vf = os.environ.get("VARIANTS_FILE")

@@ -53,10 +53,9 @@ struct TileParams {
     uint32_t *gbar;       // group-split kernel: one arrival counter per group (workspace)
     int vec16;            // generic path: tiles 16-byte aligned, 16-byte loads
     int arrive_release;   // group kernels: release-ordered arrivals (default relaxed)
-    int bulk;             // tile_group_db: slices fetched by 1-D bulk copies (TMA engine)
     int diag;             // group kernels, measurement only (IPT_TILE_DIAG; results invalid):
                           // 1 = no group wait, 2 = no stores, 4 = no loads, 32 = stores
-                          // to a second buffer after the data, 64 = evict_first loads; 16 = timeline
+                          // to a second buffer after the data; 16 = timeline
                           // trace (results valid, see ipt__tile_trace)
     unsigned long long *trace;
 };
@@ -464,6 +463,14 @@ __global__ void __launch_bounds__(512, 1) tile_onchip_stream(const TileParams p)
 // tile is signalled half-way through the current write-out, so the wait is normally
 // already satisfied (a CTA only arrives for tile i+1 after passing the wait for tile i,
 // hence the cumulative count K*(i+1) identifies tile i).
+// Memory ordering: an arrival reports that this CTA's READS of the tile have completed
+// (their data is in shared memory; the CTA observed that through the mbarrier), and the
+// waiters then WRITE the tile -- a load-buffering shape, not message passing.  A release
+// would only order this CTA's earlier *writes* (the previous tile's write-out, which no
+// waiter reads) and costs a MEMBAR.GPU that drains them: 25 % of a copy pipeline's
+// bandwidth (tools/probe_copy.py, 4.7 vs 5.9 TB/s).  So the arrival is relaxed; the
+// waiter's acquire poll keeps its stores after the observed count (stores are never
+// performed before the loop exit they depend on).  IPT_TILE_ARRIVE_RELEASE=1 restores it.
 __device__ __forceinline__ void group_arrive(uint32_t *ctr, bool release) {
     if (release) asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
     else asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
@@ -605,27 +612,6 @@ __global__ void __launch_bounds__(512, 1) tile_group_db(const TileParams p) {
     group_loop(p, s0, mbar,
         [&](const char *g, uint32_t sb) {
             const char *src = g + ((size_t)b0 * V * nvr + c0) * 16;
-            if (p.bulk) {   // one bulk copy per slice row (cvec vectors), issued by warp 0
-                if (threadIdx.x < 32) {
-                    const uint32_t sbar = smem_u32(&mbar[(sb - s0) / p.buf_bytes]);
-                    if (threadIdx.x == 0) mbar_expect_tx(&mbar[(sb - s0) / p.buf_bytes], cnt * 16);
-                    __syncwarp();
-                    for (uint32_t i = threadIdx.x; i < nb * V; i += 32)
-                        bulk_g2s_u32(sb + i * q * 16, src + (size_t)i * nvr * 16, cvec * 16, sbar);
-                }
-                return;
-            }
-            if (p.diag & 64) {
-                uint64_t pol;
-                asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-                for (uint32_t e = threadIdx.x; e < cnt; e += blockDim.x) {
-                    uint32_t i, j;
-                    fdivmod32(e, divc, i, j);
-                    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;"
-                                 :: "r"(sb + (i * q + j) * 16), "l"(src + ((size_t)i * nvr + j) * 16), "l"(pol) : "memory");
-                }
-                return;
-            }
             for (uint32_t e = threadIdx.x; e < cnt; e += blockDim.x) {
                 uint32_t i, j;
                 fdivmod32(e, divc, i, j);
@@ -1276,7 +1262,6 @@ cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, in
         p.trace = g_trace;
         if (!g_trace) p.diag &= ~16;
     }
-    p.bulk = (int)env_int("IPT_TILE_BULK", 0);
     p.arrive_release = (int)env_int("IPT_TILE_ARRIVE_RELEASE", 0);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) <= budget) {

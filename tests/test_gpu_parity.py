@@ -649,6 +649,26 @@ def test_ipt_010_group_forced_sizes(monkeypatch, K, split):
     assert np.array_equal(to_np(t, 4), oracle_P(a.copy(), batch, A, B, 1, 4)), (K, split)
 
 
+@pytest.mark.parametrize("batch,A,B", [(10, 256, 15000), (10, 7200, 240), (20, 64, 16384),
+                                       (5, 14803, 256), (6, 192, 9998)])
+def test_group_split_stress_relaxed_arrivals(batch, A, B):
+    """Stress of the group kernels' relaxed arrivals on the sweep's
+    panel tiles at full size: 24 transposes back and forth, checked against torch after an
+    odd count and against the original after an even one."""
+    import torch
+    t = torch.randint(-2**31, 2**31 - 1, (batch * A * B,), dtype=torch.int32, device="cuda")
+    orig = t.clone()
+    ref_t = orig.view(batch, A, B).transpose(1, 2).contiguous().view(-1)
+    for rep in range(24):
+        x, y = (A, B) if rep % 2 == 0 else (B, A)
+        ipt.ipt_010_(t, batch, x, y)
+        if rep == 10:
+            torch.cuda.synchronize()
+            assert torch.equal(t, ref_t), rep
+    torch.cuda.synchronize()
+    assert torch.equal(t, orig)
+
+
 _CONCURRENT_GROUPS = r"""
 import sys, torch
 sys.path.insert(0, sys.argv[1])

@@ -240,6 +240,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--queues", type=int, default=4)
+    ap.add_argument("--e2e-streams", type=int, default=2)
     ap.add_argument("--autotune", type=int, default=4,
                     help="candidates timed by ipt_plan_autotune per shape (<2: model plan)")
     ap.add_argument("--algo", default="3stage", choices=["3stage", "4stage"],
@@ -479,7 +480,7 @@ def main():
 
         # Two streams (each with its own device staging buffer): the H2D of one matrix
         # overlaps the stages and D2H of the previous one (both PCIe directions busy).
-        e2e_streams = [torch.cuda.Stream(device=dev), torch.cuda.Stream(device=dev)]
+        e2e_streams = [torch.cuda.Stream(device=dev) for _ in range(args.e2e_streams)]
 
         def e2e_step():
             cur = torch.cuda.current_stream()
@@ -487,7 +488,8 @@ def main():
                 st_.wait_stream(cur)
             for i, (h, M, N) in enumerate(hosts):
                 a, b = (N, M) if horient[i] else (M, N)
-                ipt.transpose_host_async_(h, a, b, queues=args.queues, stream=e2e_streams[i % 2])
+                ipt.transpose_host_async_(h, a, b, queues=args.queues,
+                                          stream=e2e_streams[i % len(e2e_streams)])
                 horient[i] = not horient[i]
             for st_ in e2e_streams:
                 cur.wait_stream(st_)
@@ -509,7 +511,7 @@ def main():
         e2e = {"value": round(hb * 2 * args.e2e_steps * world / (float(ems.item()) / 1e3) / 1e9, 3),
                "unit": "GB/s", "h2d_bytes_per_step": hb, "d2h_bytes_per_step": hb,
                "steps": args.e2e_steps, "queues": args.queues, "wall_s": round(wall, 3),
-               "api": "ipt_transpose_host_async on 2 streams (pinned host buffers, Sec. 6 queues)"}
+               "api": f"ipt_transpose_host_async on {len(e2e_streams)} streams (pinned host buffers, Sec. 6 queues)"}
         # verify one host result
         (h, M, N) = hosts[0]
         idx = torch.randint(0, M * N, (2048,))

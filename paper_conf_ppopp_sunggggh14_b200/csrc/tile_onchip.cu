@@ -27,6 +27,9 @@
 #include "ipt_internal.h"
 #include "mem_ptx.cuh"
 
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
 #include <cstdio>
 #include <map>
 #include <mutex>
@@ -53,6 +56,9 @@ struct TileParams {
     uint32_t *gbar;       // group-split kernel: one arrival counter per group (workspace)
     int vec16;            // generic path: tiles 16-byte aligned, 16-byte loads
     int arrive_release;   // group kernels: release-ordered arrivals (default relaxed)
+    uint32_t box_rows;    // tile_group_tma: rows per 2-D TMA box (divides the slice rows)
+    uint32_t npan;        // tile_group_tma: column panels per slice (width q vectors each)
+    uint32_t pstride;     // tile_group_tma: bytes between panels (128-byte multiple)
     int diag;             // group kernels, measurement only (IPT_TILE_DIAG; results invalid):
                           // 1 = no group wait, 2 = no stores, 4 = no loads, 32 = stores
                           // to a second buffer after the data; 16 = timeline
@@ -156,6 +162,43 @@ __device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, c
 template <int EB>
 __device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, char *g) {
     write_out<EB>(p, sbase, g, p.q, 0, p.m / (16 / EB), p.divMV32, 0, p.n / (16 / EB));
+}
+
+// As write_out, for a slice held as column panels (tile_group_tma): 16-byte column bjl
+// lives in panel bjl / pw at sbase + panel * pstride, row pitch pw vectors.
+template <int EB, typename Probe>
+__device__ __forceinline__ void write_out_pan(const TileParams &p, uint32_t sbase, char *g, uint32_t pw,
+                                              const FastDiv32 &divpw, uint32_t pstride, uint32_t bi0,
+                                              uint32_t mvp, const FastDiv32 &divmvp, uint32_t bj0,
+                                              uint32_t nbj, Probe probe) {
+    constexpr int V = 16 / EB;
+    constexpr int ROT = (V >= 8) ? 1 : 8 / V;
+    using E = typename Elem<EB>::T;
+    const uint32_t nblk = mvp * nbj;
+    for (uint32_t blk = threadIdx.x; blk < nblk; blk += blockDim.x) {
+        probe();
+        uint32_t bjl, bil, pan, pc;
+        fdivmod32(blk, divmvp, bjl, bil);
+        fdivmod32(bjl, divpw, pan, pc);
+        const uint32_t bi = bi0 + bil, bj = bj0 + bjl;
+        const int off = (int)((bil / ROT) % V);
+        const uint32_t pb = sbase + pan * pstride + pc * 16;
+        E x[V][V];
+#pragma unroll
+        for (int kk = 0; kk < V; ++kk) {
+            const uint32_t rho = (uint32_t)((kk + off) % V);
+            const uint4 v = lds128(pb + (bil * V + rho) * pw * 16);
+            unpack<EB>(v, x[kk]);
+        }
+#pragma unroll
+        for (int c = 0; c < V; ++c) {
+            E col[V];
+#pragma unroll
+            for (int kk = 0; kk < V; ++kk) col[kk] = x[kk][c];
+            rotate_sel<V, E>(col, off);
+            stg128_na(g + ((size_t)(bj * V + c) * p.m + (size_t)bi * V) * EB, pack<EB>(col));
+        }
+    }
 }
 
 // ------------------------------------------------------------------- TMA ring kernel
@@ -623,6 +666,61 @@ __global__ void __launch_bounds__(512, 1) tile_group_db(const TileParams p) {
         });
 }
 
+// --------------------------------------------------- group-split kernel, TMA slices
+// As tile_group_db, but each slice is fetched by 2-D tensor copies (cp.async.bulk.tensor,
+// the TMA engine) from a tensor map over the stacked tiles ((count*m) rows x n columns):
+// one copy per box of box_rows rows x (q*V) columns lands the slice at an odd pitch of q
+// 16-byte vectors (columns beyond n are zero-filled, columns of the neighbour slice are
+// read but never written), so no thread issues per-vector loads.
+__device__ __forceinline__ void tma_load_2d(uint32_t sdst, const CUtensorMap *tm, int32_t x, int32_t y,
+                                            uint32_t sbar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+        :: "r"(sdst), "l"(tm), "r"(x), "r"(y), "r"(sbar) : "memory");
+}
+
+template <int EB>
+__global__ void __launch_bounds__(512, 1) tile_group_tma(const TileParams p, const __grid_constant__ CUtensorMap tmap) {
+    constexpr int V = 16 / EB;
+    extern __shared__ __align__(128) unsigned char smem[];
+    const uint32_t s0 = smem_u32(smem);
+    const uint32_t K = p.K;
+    const uint32_t rank = blockIdx.x % K;
+    const uint32_t mv = p.m / V, nvr = p.n / V;
+    uint32_t b0, b1, c0, c1;
+    if (!p.colsplit) {
+        b0 = (uint32_t)((uint64_t)rank * mv / K);
+        b1 = (uint32_t)((uint64_t)(rank + 1) * mv / K);
+        c0 = 0; c1 = nvr;
+    } else {
+        b0 = 0; b1 = mv;
+        c0 = (uint32_t)((uint64_t)rank * nvr / K);
+        c1 = (uint32_t)((uint64_t)(rank + 1) * nvr / K);
+    }
+    const uint32_t q = p.q;   // panel width in vectors (odd), the same for every CTA
+    const uint32_t nb = b1 - b0, cvec = c1 - c0;
+    const uint32_t rows = p.colsplit ? p.m : (uint32_t)(((uint64_t)mv + K - 1) / K) * V;  // rows fetched
+    const uint32_t pstride = p.pstride;
+    const FastDiv32 divnb = make_fastdiv32_dev(nb), divq = make_fastdiv32_dev(q);
+    __shared__ __align__(8) uint64_t mbar[kGroupMaxBuf];
+    group_loop(p, s0, mbar,
+        [&](const char *g, uint32_t sb) {
+            if (threadIdx.x == 0) {
+                const uint64_t row0 = (uint64_t)(g - p.base) / ((uint64_t)p.n * EB) + (uint64_t)b0 * V;
+                uint64_t *bar = &mbar[(sb - s0) / p.buf_bytes];
+                mbar_expect_tx(bar, p.npan * rows * q * 16);
+                const uint32_t sbar = smem_u32(bar);
+                for (uint32_t pn = 0; pn < p.npan; ++pn)
+                    for (uint32_t r = 0; r < rows; r += p.box_rows)
+                        tma_load_2d(sb + pn * pstride + r * q * 16, &tmap, (int32_t)((c0 + pn * q) * V),
+                                    (int32_t)(row0 + r), sbar);
+            }
+        },
+        [&](char *g, uint32_t sb, auto probe) {
+            write_out_pan<EB>(p, sb, g, q, divq, pstride, b0, nb, divnb, c0, cvec, probe);
+        });
+}
+
 // ------------------------------------------------- group-split element-path kernel
 // Tiles whose sides are not multiples of 16/elem (e.g. 64 x 9998 or 14803 x 32 floats),
 // 4- and 8-byte elements, over a CTA group as tile_group_db.  A slice is a set of row
@@ -987,6 +1085,35 @@ static bool fast_colsplit(int64_t A, int64_t B, int eb) {
     return A < B && A * eb < 1024 && env_int("IPT_TILE_FAST_COLSPLIT", 1);
 }
 
+// Slice geometry of tile_group_tma: the vectors a slice row needs are fetched as npan
+// column panels of q vectors (odd, q*V <= 256 elements per box row), each as boxes of br
+// rows (br divides the fetched rows).  ok = false when the TMA path does not apply.
+struct TmaGeom {
+    bool ok = false;
+    uint32_t q = 0, npan = 0, rows = 0, br = 0;
+    size_t pstride = 0, bytes = 0;   // panel stride (128-byte aligned), slice bytes
+};
+
+static TmaGeom tma_geom(int64_t A, int64_t B, int eb, int K, bool cs) {
+    TmaGeom t;
+    if ((eb != 4 && eb != 8) || !env_int("IPT_TILE_GROUP_TMA", 1)) return t;
+    const int V = 16 / eb;
+    const int64_t mv = A / V, nvr = B / V;
+    const uint32_t need = (uint32_t)(cs ? (nvr + K - 1) / K : nvr);
+    t.rows = (uint32_t)(cs ? A : ((mv + K - 1) / K) * V);
+    const uint32_t maxw = 256 / V - 1;
+    t.npan = (need + maxw - 1) / maxw;
+    t.q = ((need + t.npan - 1) / t.npan) | 1u;
+    // box destinations must be 128-byte aligned: several boxes per panel need br % 8 == 0
+    for (uint32_t b = std::min<uint32_t>(t.rows, 256); b >= 1; --b)
+        if (t.rows % b == 0 && (b == t.rows || b % 8 == 0)) { t.br = b; break; }
+    if (t.br == 0 || (t.br < 16 && t.br != t.rows)) return t;
+    t.pstride = (((size_t)t.rows * t.q * 16) + 127) & ~(size_t)127;
+    t.bytes = (size_t)t.npan * t.pstride;
+    t.ok = true;
+    return t;
+}
+
 // Group split (tile_group_db / tile_group_generic): K CTAs per tile, `groups` tiles in
 // flight, nbuf slice buffers per CTA.  K minimises waves x (slice + 4 KB barrier
 // allowance); a larger K must win by 3 % (fewer CTAs per barrier, longer pieces).
@@ -1036,6 +1163,10 @@ static GroupCfg group_search(int64_t A, int64_t B, int eb, uint64_t count, int d
             slice = cs ? (size_t)A * (size_t)(((nvr + K - 1) / K) | 1) * 16
                        : (size_t)((mv + K - 1) / K) * V * fast_q(B, eb) * 16;
         }
+        if (!generic) {   // room for the TMA panel layout when that path applies
+            const TmaGeom t = tma_geom(A, B, eb, K, cs);
+            if (t.ok) slice = std::max(slice, t.bytes);
+        }
         slice = (slice + 127) & ~(size_t)127;
         if ((long)(nb * slice) + kGroupStaticSmem > budget) continue;
         const int64_t groups = std::min<int64_t>(dp.sms / K, (int64_t)cnt);
@@ -1070,6 +1201,52 @@ GroupCfg group_cfg_generic(int64_t A, int64_t B, int eb, uint64_t count, int dev
     return group_choose(A, B, eb, count, device, true);
 }
 
+// Tensor map + box geometry for tile_group_tma (IPT_TILE_GROUP_TMA, default on): 4- and 8-byte elements,
+// tiles stacked contiguously, a uniform odd box width of at most 256 elements, and a box
+// height dividing the fetched slice rows.  Returns false when the TMA path does not apply.
+static PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        cudaDriverEntryPointQueryResult q;
+        void *f = nullptr;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (PFN_cuTensorMapEncodeTiled_v12000)f;
+    });
+    return fn;
+}
+
+template <int EB>
+bool group_tma_setup(const StageDesc &d, TileParams &p, const GroupCfg &g, CUtensorMap *tm) {
+    if (EB != 4 && EB != 8) return false;
+    if (d.outer > 1 && d.ostride != d.inner * (int64_t)p.tile_bytes) return false;
+    const TmaGeom t = tma_geom(d.A, d.B, EB, g.K, g.colsplit);
+    if (!t.ok || t.bytes > g.slice) return false;
+    auto enc = tensor_map_encoder();
+    if (!enc) return false;
+    const int V = 16 / EB;
+    const uint64_t total_rows = (uint64_t)(d.outer * d.inner) * (uint64_t)d.A;
+    cuuint64_t dims[2] = {(cuuint64_t)d.B, (cuuint64_t)total_rows};
+    cuuint64_t strides[1] = {(cuuint64_t)(d.B * EB)};
+    cuuint32_t box[2] = {t.q * V, t.br};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(tm, EB == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 2, d.base,
+                     dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) {
+        if (env_int("IPT_DEBUG", 0)) fprintf(stderr, "[ipt] tensor map encode failed (%d)\n", (int)r);
+        return false;
+    }
+    p.q = t.q;
+    p.box_rows = t.br;
+    p.npan = t.npan;
+    p.pstride = (uint32_t)t.pstride;
+    if (env_int("IPT_DEBUG", 0))
+        fprintf(stderr, "[ipt] tile_group_tma q=%u npan=%u rows=%u box=%ux%u\n", t.q, t.npan, t.rows, t.q * V, t.br);
+    return true;
+}
+
 // Group-split launch: groups x K CTAs, all co-resident (cooperative launch); the arrival
 // counters (workspace, kGroupCtrStride bytes apart) are zeroed on the stream first.
 template <int EB, bool GENERIC>
@@ -1089,20 +1266,24 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
     p.gbar = (uint32_t *)ws;
     if ((size_t)g.groups * g.nbuf * kGroupCtrStride > kTileWsBytes) return cudaErrorInvalidValue;
     auto kern = GENERIC ? tile_group_generic<EB> : tile_group_db<EB>;
+    CUtensorMap tmap;
+    const bool tma = !GENERIC && group_tma_setup<EB>(d, p, g, &tmap);
     cudaError_t e = cudaMemsetAsync(ws, 0, (size_t)g.groups * g.nbuf * kGroupCtrStride, st);
     if (e != cudaSuccess) return e;
-    {   // dynamic + static shared memory must stay within the opt-in maximum
+    auto set_smem = [&](const void *k) {   // dynamic + static shared memory within the opt-in maximum
         static std::mutex mu;
         static std::map<std::pair<const void *, int>, bool> done;
         std::lock_guard<std::mutex> lk(mu);
-        if (!done[std::make_pair((const void *)kern, device)]) {
+        if (!done[std::make_pair(k, device)]) {
             cudaFuncAttributes fa{};
-            cudaFuncGetAttributes(&fa, kern);
-            cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+            cudaFuncGetAttributes(&fa, k);
+            cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  dev_props(device).smem_optin - (int)fa.sharedSizeBytes);
-            done[std::make_pair((const void *)kern, device)] = true;
+            done[std::make_pair(k, device)] = true;
         }
-    }
+    };
+    set_smem((const void *)kern);
+    if (tma) set_smem((const void *)tile_group_tma<EB>);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)(g.groups * g.K), 1, 1);
     cfg.blockDim = dim3(512, 1, 1);
@@ -1117,7 +1298,7 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
         fprintf(stderr, "[ipt] tile_group%s m=%u n=%u K=%d groups=%d colsplit=%d smem=%zu tiles=%llu\n",
                 GENERIC ? "_generic" : "", p.m, p.n, g.K, g.groups, p.colsplit, g.nbuf * g.slice,
                 (unsigned long long)p.count);
-    e = cudaLaunchKernelEx(&cfg, kern, p);
+    e = tma ? cudaLaunchKernelEx(&cfg, tile_group_tma<EB>, p, tmap) : cudaLaunchKernelEx(&cfg, kern, p);
     note_launch();
     return e != cudaSuccess ? e : cudaGetLastError();
 }

@@ -649,6 +649,22 @@ def test_ipt_010_group_forced_sizes(monkeypatch, K, split):
     assert np.array_equal(to_np(t, 4), oracle_P(a.copy(), batch, A, B, 1, 4)), (K, split)
 
 
+@pytest.mark.parametrize("tma", ["0", "1"])
+@pytest.mark.parametrize("eb,batch,A,B,K", [(4, 3, 64, 16384, "0"), (4, 2, 384, 10000, "0"), (4, 3, 7200, 240, "0"),
+                                            (4, 2, 10000, 384, "0"), (4, 2, 7200, 240, "71"), (4, 2, 240, 7200, "33"),
+                                            (8, 2, 3000, 200, "0"), (8, 2, 200, 3000, "0"), (8, 1, 600, 6000, "0")])
+def test_ipt_010_group_tma_slices(monkeypatch, tma, eb, batch, A, B, K):
+    """Group tiles with slices fetched by 2-D TMA boxes: one or two column panels, several
+    row boxes per panel, uneven row slices (the boxes read the neighbour's rows), f64 --
+    and the same shapes on the cp.async path."""
+    monkeypatch.setenv("IPT_TILE_GROUP_TMA", tma)
+    monkeypatch.setenv("IPT_TILE_GROUP_K", K)
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (tma, eb, batch, A, B, K)
+
+
 @pytest.mark.parametrize("batch,A,B", [(10, 256, 15000), (10, 7200, 240), (20, 64, 16384),
                                        (5, 14803, 256), (6, 192, 9998)])
 def test_group_split_stress_relaxed_arrivals(batch, A, B):

@@ -97,7 +97,8 @@ int tile_generic_cluster_k(int64_t A, int64_t B, int eb, int device);
 bool tile_group_split(int64_t A, int64_t B, int eb, int device);
 bool tile_group_generic_split(int64_t A, int64_t B, int eb, int device);
 // Group split of `count` tiles: CTAs per tile (0 = does not fit) and groups in flight.
-int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups);
+int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups,
+                 bool *tma = nullptr);
 // Workspace of a tile stage: the group split's arrival counters (one per group and slice
 // buffer, kGroupCtrStride bytes apart, at most 256).  `ws` may be NULL for the other paths.
 constexpr uint32_t kGroupCtrStride = 32;

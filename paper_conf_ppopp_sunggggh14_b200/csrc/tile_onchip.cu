@@ -1400,10 +1400,12 @@ bool tile_group_generic_split(int64_t A, int64_t B, int eb, int device) {
     return group_cfg_generic(A, B, eb, (uint64_t)dev_props(device).sms, device).K != 0;
 }
 
-int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups) {
-    const GroupCfg g = vec_ok(A, B, eb) ? group_cfg(A, B, eb, count, device)
-                                        : group_cfg_generic(A, B, eb, count, device);
+int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups, bool *tma) {
+    const bool fast = vec_ok(A, B, eb);
+    const GroupCfg g = fast ? group_cfg(A, B, eb, count, device)
+                            : group_cfg_generic(A, B, eb, count, device);
     if (groups) *groups = g.groups;
+    if (tma) *tma = fast && g.K && tma_geom(A, B, eb, g.K, g.colsplit).ok;
     return g.K;
 }
 

@@ -365,6 +365,10 @@ def main():
             step_ev[s][0].record()
             one_step(evs[s] if args.algo == "3stage" else None)
             step_ev[s][1].record()
+    # wait with the GIL released so the clock sampler thread runs during the whole region
+    last = t_end if flush is None else step_ev[-1][1]
+    while not last.query():
+        time.sleep(0.0005)
     torch.cuda.synchronize()
     torch.cuda.nvtx.range_pop()
     launches = ipt.kernel_launch_count() - launches0

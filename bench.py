@@ -240,7 +240,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--queues", type=int, default=4)
-    ap.add_argument("--e2e-streams", type=int, default=2)
+    ap.add_argument("--e2e-streams", type=int, default=4)
     ap.add_argument("--autotune", type=int, default=4,
                     help="candidates timed by ipt_plan_autotune per shape (<2: model plan)")
     ap.add_argument("--algo", default="3stage", choices=["3stage", "4stage"],
@@ -482,7 +482,7 @@ def main():
         torch.cuda.empty_cache()
         horient = [False] * len(hosts)
 
-        # Two streams (each with its own device staging buffer): the H2D of one matrix
+        # Several streams (each with its own device staging buffer): the H2D of one matrix
         # overlaps the stages and D2H of the previous one (both PCIe directions busy).
         e2e_streams = [torch.cuda.Stream(device=dev) for _ in range(args.e2e_streams)]
 

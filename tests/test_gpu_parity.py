@@ -665,6 +665,20 @@ def test_ipt_010_group_tma_slices(monkeypatch, tma, eb, batch, A, B, K):
     assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (tma, eb, batch, A, B, K)
 
 
+@pytest.mark.parametrize("eb,batch,A,B,K", [(4, 2, 128, 9998, "0"), (4, 2, 9998, 128, "0"), (4, 1, 256, 14803, "0"),
+                                            (4, 1, 14803, 256, "0"), (4, 2, 192, 9998, "0"), (4, 3, 601, 1203, "5"),
+                                            (8, 2, 3001, 62, "0"), (8, 2, 62, 3001, "7"), (4, 2, 1998, 130, "9")])
+def test_ipt_010_group_tma_element_slices(monkeypatch, eb, batch, A, B, K):
+    """Element-path group tiles with TMA slices (opt-in path): rows grouped R = 1, 2, 4 per
+    super-row, per-class phases realigned on write-out, one or two panels."""
+    monkeypatch.setenv("IPT_TILE_GROUP_TMA_GENERIC", "1")
+    monkeypatch.setenv("IPT_TILE_GROUP_K", K)
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B, K)
+
+
 @pytest.mark.parametrize("batch,A,B", [(10, 256, 15000), (10, 7200, 240), (20, 64, 16384),
                                        (5, 14803, 256), (6, 192, 9998)])
 def test_group_split_stress_relaxed_arrivals(batch, A, B):

@@ -68,7 +68,10 @@ typedef enum {
     IPT_VAR_IDENTITY = 0,      /* stage elided: a swapped dimension is 1 */
     IPT_VAR_TILE_ONCHIP = 1,   /* whole tile staged in shared memory (BS, Fig. 1) */
     IPT_VAR_CYCLE_ONCHIP = 2,  /* PTTWAC inside a tile, flag bits in shared memory */
-    IPT_VAR_CYCLE_GLOBAL = 3   /* PTTWAC over super-elements, flag bits in global memory */
+    IPT_VAR_CYCLE_GLOBAL = 3,  /* PTTWAC over super-elements, flag bits in global memory */
+    IPT_VAR_SQUARE_SWAP = 4    /* square tiles (m == n, any size): symmetric swaps across the
+                                  diagonal, cycles of length 2; with m = M = N = n the
+                                  whole transposition is this single pass */
 } ipt_variant;
 
 /* A plan for the 3-stage transposition of one M x N matrix (Sec. 4.2 + Sec. 7.4). */

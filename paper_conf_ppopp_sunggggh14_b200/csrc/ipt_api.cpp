@@ -202,8 +202,11 @@ ipt_status validate_plan(const ipt_plan_t *p) {
         p->Np != p->N / p->n)
         return IPT_ERR_INVALID_ARG;
     for (int i = 0; i < 3; ++i)
-        if (p->variant[i] < IPT_VAR_IDENTITY || p->variant[i] > IPT_VAR_CYCLE_GLOBAL)
+        if (p->variant[i] < IPT_VAR_IDENTITY || p->variant[i] > IPT_VAR_SQUARE_SWAP)
             return IPT_ERR_INVALID_ARG;
+    if ((p->variant[0] == IPT_VAR_SQUARE_SWAP || p->variant[2] == IPT_VAR_SQUARE_SWAP) ||
+        (p->variant[1] == IPT_VAR_SQUARE_SWAP && p->m != p->n))
+        return IPT_ERR_INVALID_ARG;   // only stage 2 with square tiles is a swap
     return IPT_OK;
 }
 
@@ -237,6 +240,7 @@ ipt_status run_plan(char *base, int64_t count, int64_t stride, const ipt_plan_t 
         switch (p->variant[i]) {
             case IPT_VAR_IDENTITY: break;
             case IPT_VAR_TILE_ONCHIP: e = launch_tile_onchip(sd[i], ws, st, device); break;
+            case IPT_VAR_SQUARE_SWAP: e = launch_square_swap(sd[i], st, device); break;
             case IPT_VAR_CYCLE_ONCHIP:   // not built yet: global-flag cycle following
             case IPT_VAR_CYCLE_GLOBAL: e = launch_cycle_global(sd[i], ws, st, device); break;
         }
@@ -403,6 +407,10 @@ ipt_status ipt_010(void *d_ptr, int64_t batch, int64_t A, int64_t B, int elem_by
     if (batch == 0 || A == 1 || B == 1) return IPT_OK;
     const int device = current_device();
     if (device < 0) return IPT_ERR_NO_DEVICE;
+    if (A == B && prefer_square_swap(batch, A, elem_bytes, device)) {   // P:45, no workspace
+        StageDesc sd = stage_desc(d_ptr, batch, A, B, 1, elem_bytes);
+        return cuda_status(launch_square_swap(sd, (cudaStream_t)stream, device));
+    }
     if (tile_onchip_fits(A, B, elem_bytes, device)) {
         StageDesc sd = stage_desc(d_ptr, batch, A, B, 1, elem_bytes);
         void *ws = d_workspace;
@@ -535,10 +543,14 @@ ipt_status ipt_transpose_4stage(void *d_ptr, int64_t M, int64_t N, int64_t m, in
     sd[2].outer = 1;       sd[2].A = Mp; sd[2].B = Np; sd[2].s = m * n;
     sd[3].outer = Np;      sd[3].A = Mp; sd[3].B = n;  sd[3].s = m;
     size_t need = 0;
-    bool tile2 = false;
+    bool tile2 = false, sq2 = false;
     for (int i = 0; i < 4; ++i) {
         sd[i].ostride = sd[i].A * sd[i].B * sd[i].s * elem_bytes;
         if (sd[i].A == 1 || sd[i].B == 1) continue;
+        if (i == 1 && m == n && prefer_square_swap(Mp * Np, m, elem_bytes, device)) {
+            sq2 = true;
+            continue;
+        }
         if (i == 1 && tile_onchip_fits(m, n, elem_bytes, device)) {
             tile2 = true;
             need = std::max(need, kTileWsBytes);
@@ -554,8 +566,9 @@ ipt_status ipt_transpose_4stage(void *d_ptr, int64_t M, int64_t N, int64_t m, in
     }
     for (int i = 0; i < 4; ++i) {
         if (sd[i].A == 1 || sd[i].B == 1) continue;
-        cudaError_t e = (i == 1 && tile2) ? launch_tile_onchip(sd[i], ws, (cudaStream_t)stream, device)
-                                          : launch_cycle_global(sd[i], ws, (cudaStream_t)stream, device);
+        cudaError_t e = (i == 1 && sq2)     ? launch_square_swap(sd[i], (cudaStream_t)stream, device)
+                        : (i == 1 && tile2) ? launch_tile_onchip(sd[i], ws, (cudaStream_t)stream, device)
+                                            : launch_cycle_global(sd[i], ws, (cudaStream_t)stream, device);
         if (e != cudaSuccess) return cuda_status(e);
     }
     return IPT_OK;
@@ -660,6 +673,7 @@ static ipt_status transpose_host_impl(void *h_ptr, int64_t M, int64_t N, int ele
         a.base = gb; a.inner = np_g * p.Mp;
         b.base = gb; b.inner = np_g;
         if (p.variant[1] == IPT_VAR_TILE_ONCHIP) e = launch_tile_onchip(a, dwsg[g], qs_g, device);
+        else if (p.variant[1] == IPT_VAR_SQUARE_SWAP) e = launch_square_swap(a, qs_g, device);
         else if (p.variant[1] == IPT_VAR_CYCLE_GLOBAL) e = launch_cycle_global(a, dwsg[g], qs_g, device);
         if (e != cudaSuccess) return cuda_status(e);
         if (p.variant[2] == IPT_VAR_CYCLE_GLOBAL) e = launch_cycle_global(b, dwsg[g], qs_g, device);

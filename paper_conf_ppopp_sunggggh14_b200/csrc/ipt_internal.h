@@ -105,6 +105,12 @@ constexpr uint32_t kGroupCtrStride = 32;
 constexpr size_t kTileWsBytes = 256 * kGroupCtrStride;
 cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, int device);
 
+// Square items P(batch, g, g, 1) by symmetric block-pair swaps: any g, no
+// workspace.  square_swap_vec_path: the 16-byte path applies (else the element path).
+cudaError_t launch_square_swap(const StageDesc &d, cudaStream_t st, int device);
+bool square_swap_vec_path(const StageDesc &d);
+bool prefer_square_swap(int64_t batch, int64_t g, int eb, int device);   // plan.cpp
+
 // Device properties used by planner and launchers (cached).
 struct DevProps {
     int sms;

@@ -143,7 +143,7 @@ def test_plan_overhead_below_paper_bound():
 
 def test_plan_prefers_vector_tiles_on_large_f32():
     """Sec. 7.4 pruning: big super-elements for stages 1/3, tile on chip for stage 2."""
-    for (M, N) in [(16384, 16384), (20000, 20000), (12800, 15000)]:
+    for (M, N) in [(12800, 15000), (15000, 12800), (19200, 10000)]:
         p = ipt.plan(M, N, 4)
         assert p.n * 4 >= 256 and p.m * 4 >= 256
         assert p.n * 4 % 16 == 0 and p.m * 4 % 16 == 0     # 16-byte vector super-elements
@@ -168,7 +168,7 @@ def test_group_split_extends_on_chip_tiles():
     ~148 x 113 KB, double-buffered); larger tiles fall back to cycle following.  A tile
     stage reserves 8 KB of workspace for the group counters (nominal B200, no GPU)."""
     V = ipt.VARIANTS
-    for (M, N, m, n) in [(4096, 4096, 1024, 1024),     # 4 MB 16-byte-path tiles
+    for (M, N, m, n) in [(4096, 8192, 1024, 1024 + 1024),  # 8 MB 16-byte-path tiles
                          (16384, 16384, 128, 16384),   # 8 MB panels (n = N)
                          (14803, 8192, 14803, 128),    # 7.6 MB element-path panels (m = M)
                          (12288, 9998, 192, 9998)]:
@@ -179,3 +179,32 @@ def test_group_split_extends_on_chip_tiles():
     assert V[p.variant[1]] == "cycle_global"
     assert ipt.lib().ipt_stage_workspace_bytes(3, 120, 7200, 1, 4) >= 8192
     assert ipt.lib().ipt_stage_workspace_bytes(1, 4, 4, 5, 4) < 8192   # cycle stage: flags only
+
+
+def test_square_matrices_plan_single_swap_pass():
+    """a square matrix is transposed by swapping symmetric elements (cycles of length
+    2) -- the planner makes it one stage, stage 2 with the whole matrix as one square tile
+    executed by the swap kernel (no flags, no workspace), for any side incl. primes."""
+    V = ipt.VARIANTS
+    for M in [1000, 2048, 4096, 10007, 16384, 20000]:
+        for eb in (4, 8, 16):
+            if M * M * eb <= (1 << 22):   # small squares may stay on chip (one CTA group)
+                continue
+            p = ipt.plan(M, M, eb)
+            assert (p.m, p.n, p.n_stages) == (M, M, 1), (M, eb)
+            assert [V[v] for v in p.variant] == ["identity", "square_swap", "identity"]
+            assert p.workspace_bytes == 0
+    # rectangular shapes never get a swap stage unless their tiles are square
+    for (M, N) in [(7200, 18000), (9998, 12288), (1_000_000, 256), (4096, 3000)]:
+        p = ipt.plan(M, N, 4)
+        assert V[p.variant[1]] != "square_swap" or p.m == p.n
+
+
+def test_forced_square_tiles_plan_validation():
+    """Square stage-2 tiles may be forced (m = n | gcd(M, N)); a hand-made plan with a swap
+    stage on non-square tiles is rejected before any launch."""
+    p = ipt.plan(7200, 1800, 4, m=1800, n=1800)
+    assert ipt.VARIANTS[p.variant[1]] in ("square_swap", "tile_onchip")
+    q = ipt.plan(7200, 1800, 4, m=120, n=200)
+    q.variant[1] = 4
+    assert ipt.lib().ipt_workspace_bytes(ctypes.byref(q), 1) == 0   # invalid plan -> 0

@@ -763,3 +763,96 @@ def test_ipt_010_group_element_misaligned_base():
     ref = a.copy()
     ref[1:] = oracle_P(a[1:].copy(), batch, A, B, 1, 4)
     assert np.array_equal(to_np(t, 4), ref)
+
+
+# ------------------------------------------- square items: symmetric swaps
+SQ_SIDES = [2, 3, 7, 15, 16, 17, 63, 64, 65, 100, 127, 128, 129, 255, 256, 257, 300, 1021]
+
+
+@pytest.mark.parametrize("eb", [1, 2, 4, 8, 16])
+@pytest.mark.parametrize("path", ["auto", "elem", "tb512"])
+def test_square_swap_sides(monkeypatch, eb, path):
+    """ipt_010 on square items through the swap kernel: every side spans ragged block
+    edges (g not a multiple of the 256-byte block) and, for g % (16/b) != 0, the element
+    path; batches fold several items into one launch."""
+    monkeypatch.setenv("IPT_SQ_FORCE", "1")
+    if path == "elem":
+        monkeypatch.setenv("IPT_SQ_ELEM", "1")
+    if path == "tb512":
+        monkeypatch.setenv("IPT_SQ_TB", "512")
+    rnd = random.Random(eb * 7 + len(path))
+    for g in SQ_SIDES:
+        batch = rnd.choice([1, 1, 2, 3]) if g > 256 else rnd.choice([1, 2, 5, 17])
+        a = gen(batch * g * g, eb)
+        t = to_dev(a, eb)
+        ipt.ipt_010_(t, batch, g, g, elem_bytes=eb)
+        ref = oracle_P(a.copy(), batch, g, g, 1, eb)
+        assert np.array_equal(to_np(t, eb), ref), (batch, g, eb, path)
+
+
+def test_square_swap_misaligned_base(monkeypatch):
+    """A base 4 bytes off 16-byte alignment takes the element path; neighbours untouched."""
+    monkeypatch.setenv("IPT_SQ_FORCE", "1")
+    batch, g = 3, 200
+    a = gen(batch * g * g + 3, 4)
+    t = to_dev(a, 4)
+    ipt.ipt_010_(t[1:1 + batch * g * g], batch, g, g)
+    got = to_np(t, 4)
+    assert got[0] == a.view(np.uint32)[0] and np.array_equal(got[-2:], a.view(np.uint32)[-2:])
+    ref = oracle_P(a[1:1 + batch * g * g].copy(), batch, g, g, 1, 4)
+    assert np.array_equal(got[1:1 + batch * g * g], ref)
+
+
+@pytest.mark.parametrize("M,eb", [(2, 4), (5, 8), (64, 4), (1000, 4), (1024, 8), (2049, 4),
+                                  (4096, 4), (997, 8)])
+def test_square_matrix_single_pass_plan(M, eb):
+    """M == N plans run one stage (square_swap) and match the oracle bit for bit."""
+    p = ipt.plan(M, M, eb, 0)
+    assert p.n_stages == 1 and ipt.VARIANTS[p.variant[1]] == "square_swap", p.as_dict()
+    a = seeded.matrix_np(M, M, eb)
+    t = to_dev(a, eb)
+    before = ipt.kernel_launch_count()
+    ipt.transpose_(t, M, M)
+    torch.cuda.synchronize()
+    assert ipt.kernel_launch_count() - before == 1
+    assert np.array_equal(to_np(t, eb), oracle.transpose_inplace(a.copy(), M, M)), (M, eb)
+
+
+def test_square_batched_with_stride():
+    """A batch of square matrices with a gap between them: gaps untouched."""
+    count, M, gap = 5, 384, 40
+    stride = M * M + gap
+    a = gen(count * stride, 4)
+    t = to_dev(a, 4)
+    ipt.transpose_batched_(t, count, M, M, stride_elems=stride)
+    got = to_np(t, 4)
+    src = a.view(np.uint32)
+    for k in range(count):
+        blk = src[k * stride:k * stride + M * M].copy()
+        assert np.array_equal(got[k * stride:k * stride + M * M],
+                              oracle.transpose_inplace(blk, M, M)), k
+        assert np.array_equal(got[k * stride + M * M:(k + 1) * stride],
+                              src[k * stride + M * M:(k + 1) * stride])
+
+
+@pytest.mark.parametrize("M,N,m", [(7200, 1800, 1800), (1800, 7200, 1800), (4096, 4096, 1024),
+                                   (3000, 6000, 1000), (640, 960, 320)])
+def test_square_tiles_in_3stage_plan(monkeypatch, M, N, m):
+    """Plans with square stage-2 tiles m = n of any size (up to 13 MB here) run stage 2
+    with the swap kernel inside the 3-stage method."""
+    monkeypatch.setenv("IPT_SQ_FORCE", "1")
+    p = ipt.plan(M, N, 4, 0, m=m, n=m)
+    assert ipt.VARIANTS[p.variant[1]] == "square_swap", p.as_dict()
+    a = seeded.matrix_np(M, N, 4)
+    t = to_dev(a, 4)
+    ipt.transpose_(t, M, N, plan_=p)
+    assert np.array_equal(to_np(t, 4), oracle.transpose_inplace(a.copy(), M, N)), (M, N, m)
+
+
+def test_square_host_path():
+    """The host-delegated scheme (Sec. 6) on a square matrix (single-pass plan)."""
+    M = 1536
+    a = seeded.matrix_np(M, M, 4)
+    h = torch.from_numpy(a.view(np.int32).copy()).pin_memory()
+    ipt.transpose_host_(h, M, M, queues=2)
+    assert np.array_equal(h.numpy().view(np.uint32), oracle.transpose_inplace(a.copy(), M, M))

@@ -395,9 +395,9 @@ def main():
     peak, peak_src = load_peaks()
 
     # ---- per-stage (per-kernel) live timing -> roofline of the dominant kernel
-    kern_t = {"cycle_global": 0.0, "tile_onchip": 0.0}
-    kern_bytes = {"cycle_global": 0, "tile_onchip": 0}
-    kern_n = {"cycle_global": 0, "tile_onchip": 0}
+    kern_t = {"cycle_global": 0.0, "tile_onchip": 0.0, "square_swap": 0.0}
+    kern_bytes = {"cycle_global": 0, "tile_onchip": 0, "square_swap": 0}
+    kern_n = {"cycle_global": 0, "tile_onchip": 0, "square_swap": 0}
     stage_scaled = None
     per_shape = {}
     if args.algo == "3stage":

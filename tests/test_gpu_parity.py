@@ -805,14 +805,19 @@ def test_square_swap_misaligned_base(monkeypatch):
 
 @pytest.mark.parametrize("M,eb", [(2, 4), (5, 8), (64, 4), (1000, 4), (1024, 8), (2049, 4),
                                   (4096, 4), (997, 8)])
-def test_square_matrix_single_pass_plan(M, eb):
-    """M == N plans run one stage (square_swap) and match the oracle bit for bit."""
-    p = ipt.plan(M, M, eb, 0)
+def test_square_matrix_single_pass_plan(monkeypatch, M, eb):
+    """M == N plans run one stage (square_swap; forced for the small sides, which the
+    planner may keep on chip) and match the oracle bit for bit."""
+    monkeypatch.setenv("IPT_SQ_FORCE", "1")
+    p = ipt.plan(M, M, eb, 0, m=M, n=M)
     assert p.n_stages == 1 and ipt.VARIANTS[p.variant[1]] == "square_swap", p.as_dict()
+    if M * M * eb > (1 << 22):
+        q = ipt.plan(M, M, eb, 0)
+        assert (q.m, q.n, list(q.variant)) == (p.m, p.n, list(p.variant))
     a = seeded.matrix_np(M, M, eb)
     t = to_dev(a, eb)
     before = ipt.kernel_launch_count()
-    ipt.transpose_(t, M, M)
+    ipt.transpose_(t, M, M, plan_=p)
     torch.cuda.synchronize()
     assert ipt.kernel_launch_count() - before == 1
     assert np.array_equal(to_np(t, eb), oracle.transpose_inplace(a.copy(), M, M)), (M, eb)

@@ -139,6 +139,8 @@ def _dev_ptr(t):
 def _events_arr(events):
     arr = (ctypes.c_void_p * 4)()
     for i, e in enumerate(events or []):
+        if e is not None and not e.cuda_event:
+            e.record()   # torch creates the cudaEvent_t lazily, on its first record
         arr[i] = ctypes.c_void_p(e.cuda_event) if e is not None else None
     return arr
 

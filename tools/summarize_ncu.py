@@ -28,6 +28,8 @@ def kind(name: str):
         return "cycle_global"
     if "tile_" in name:
         return "tile_onchip"
+    if "square_swap" in name:
+        return "square_swap"
     return None
 
 
@@ -97,7 +99,8 @@ WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
 
 
 def full(tag):
-    out = [f"# {tag}: ncu --set full captures (`tools/prof_one.py 12800 15000`)", ""]
+    out = [f"# {tag}: ncu --set full captures (`tools/prof_one.py 12800 15000`, 9998 12288, "
+           "16384 16384 for square_swap)", ""]
     for rep in sorted(f for f in os.listdir(GO) if f.startswith("prof_") and f.endswith(".ncu-rep")):
         raw = subprocess.run([NCU, "-i", os.path.join(GO, rep), "--page", "raw", "--csv"],
                              capture_output=True, text=True).stdout

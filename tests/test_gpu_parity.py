@@ -770,16 +770,19 @@ SQ_SIDES = [2, 3, 7, 15, 16, 17, 63, 64, 65, 100, 127, 128, 129, 255, 256, 257, 
 
 
 @pytest.mark.parametrize("eb", [1, 2, 4, 8, 16])
-@pytest.mark.parametrize("path", ["auto", "elem", "tb512"])
+@pytest.mark.parametrize("path", ["auto", "vec", "elem", "tb512"])
 def test_square_swap_sides(monkeypatch, eb, path):
-    """ipt_010 on square items through the swap kernel: every side spans ragged block
-    edges (g not a multiple of the 256-byte block) and, for g % (16/b) != 0, the element
-    path; batches fold several items into one launch."""
+    """ipt_010 on square items through the swap kernel (TMA ring by default, register
+    staged, element path): every side spans ragged block edges (g not a multiple of the
+    block) and, for g % (16/b) != 0, the element path; batches fold several items into
+    one launch (rows of a ragged last block belong to the next item)."""
     monkeypatch.setenv("IPT_SQ_FORCE", "1")
     if path == "elem":
         monkeypatch.setenv("IPT_SQ_ELEM", "1")
     if path == "tb512":
         monkeypatch.setenv("IPT_SQ_TB", "512")
+    if path in ("vec", "tb512"):
+        monkeypatch.setenv("IPT_SQ_TMA", "0")
     rnd = random.Random(eb * 7 + len(path))
     for g in SQ_SIDES:
         batch = rnd.choice([1, 1, 2, 3]) if g > 256 else rnd.choice([1, 2, 5, 17])
@@ -861,3 +864,30 @@ def test_square_host_path():
     h = torch.from_numpy(a.view(np.int32).copy()).pin_memory()
     ipt.transpose_host_(h, M, M, queues=2)
     assert np.array_equal(h.numpy().view(np.uint32), oracle.transpose_inplace(a.copy(), M, M))
+
+
+@pytest.mark.parametrize("nb", [2, 3, 7])
+def test_square_swap_tma_ring_depths(monkeypatch, nb):
+    """The TMA ring wraps many times (phase parity of full/empty barriers) at small depths."""
+    monkeypatch.setenv("IPT_SQ_FORCE", "1")
+    monkeypatch.setenv("IPT_SQ_NB", str(nb))
+    for (batch, g, eb) in [(3, 1000, 4), (2, 777 * 2, 8), (40, 129, 4), (5, 96, 16)]:
+        a = gen(batch * g * g, eb)
+        t = to_dev(a, eb)
+        ipt.ipt_010_(t, batch, g, g, elem_bytes=eb)
+        assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, g, g, 1, eb)), (batch, g, eb)
+
+
+def test_square_swap_strided_batch_tma(monkeypatch):
+    """3-D tensor map: outer items at a stride (a gap after every item) -- gaps untouched."""
+    count, M, gap = 4, 1000, 4 * 7
+    stride = M * M + gap
+    a = gen(count * stride, 4)
+    t = to_dev(a, 4)
+    ipt.transpose_batched_(t, count, M, M, stride_elems=stride)
+    got = to_np(t, 4)
+    src = a.view(np.uint32)
+    for k in range(count):
+        blk = src[k * stride:k * stride + M * M].copy()
+        assert np.array_equal(got[k * stride:k * stride + M * M], oracle.transpose_inplace(blk, M, M)), k
+        assert np.array_equal(got[k * stride + M * M:(k + 1) * stride], src[k * stride + M * M:(k + 1) * stride])

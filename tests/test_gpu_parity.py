@@ -770,7 +770,7 @@ SQ_SIDES = [2, 3, 7, 15, 16, 17, 63, 64, 65, 100, 127, 128, 129, 255, 256, 257, 
 
 
 @pytest.mark.parametrize("eb", [1, 2, 4, 8, 16])
-@pytest.mark.parametrize("path", ["auto", "vec", "elem", "tb512"])
+@pytest.mark.parametrize("path", ["auto", "tma", "vec", "elem", "tb512"])
 def test_square_swap_sides(monkeypatch, eb, path):
     """ipt_010 on square items through the swap kernel (TMA ring by default, register
     staged, element path): every side spans ragged block edges (g not a multiple of the
@@ -783,6 +783,8 @@ def test_square_swap_sides(monkeypatch, eb, path):
         monkeypatch.setenv("IPT_SQ_TB", "512")
     if path in ("vec", "tb512"):
         monkeypatch.setenv("IPT_SQ_TMA", "0")
+    if path == "tma":
+        monkeypatch.setenv("IPT_SQ_TMA", "1")
     rnd = random.Random(eb * 7 + len(path))
     for g in SQ_SIDES:
         batch = rnd.choice([1, 1, 2, 3]) if g > 256 else rnd.choice([1, 2, 5, 17])
@@ -866,11 +868,16 @@ def test_square_host_path():
     assert np.array_equal(h.numpy().view(np.uint32), oracle.transpose_inplace(a.copy(), M, M))
 
 
-@pytest.mark.parametrize("nb", [2, 3, 7])
-def test_square_swap_tma_ring_depths(monkeypatch, nb):
-    """The TMA ring wraps many times (phase parity of full/empty barriers) at small depths."""
+@pytest.mark.parametrize("nb,st,tma", [(2, 0, 1), (3, 2, 1), (7, 1, 1), (0, 3, 1), (0, 2, 0),
+                                       (0, 1, 0), (0, 0, 0)])
+def test_square_swap_tma_ring_depths(monkeypatch, nb, st, tma):
+    """The TMA ring wraps many times (phase parity of full/empty barriers) at small depths;
+    super-tile pair orders (S = 2^st, empty slots below the diagonal and past the edge)
+    on both the TMA and the register-staged kernels."""
     monkeypatch.setenv("IPT_SQ_FORCE", "1")
     monkeypatch.setenv("IPT_SQ_NB", str(nb))
+    monkeypatch.setenv("IPT_SQ_ST", str(st))
+    monkeypatch.setenv("IPT_SQ_TMA", str(tma))
     for (batch, g, eb) in [(3, 1000, 4), (2, 777 * 2, 8), (40, 129, 4), (5, 96, 16)]:
         a = gen(batch * g * g, eb)
         t = to_dev(a, eb)

@@ -7,21 +7,22 @@ if os.environ.get("_CHILD"):
     import torch
     import paper_conf_ppopp_sunggggh14_b200 as ipt
     TOT_BYTES = 800 << 20
-    dt = {4: torch.int32, 8: torch.int64}
+    dt = {4: torch.int32, 8: torch.int64, 16: torch.int64}
     res = {}
     for (g, eb) in ast.literal_eval(os.environ["SHAPES"]):
         cnt = max(1, TOT_BYTES // (g * g * eb))
-        buf = torch.empty(cnt * g * g, dtype=dt[eb], device="cuda")
+        w = 2 if eb == 16 else 1
+        buf = torch.empty(cnt * g * g * w, dtype=dt[eb], device="cuda")
         buf.random_()
-        ref = buf.view(cnt, g, g).transpose(1, 2).contiguous().view(-1)
-        ipt.ipt_010_(buf, cnt, g, g)
+        ref = buf.view(cnt, g, g, w).transpose(1, 2).contiguous().view(-1)
+        ipt.ipt_010_(buf, cnt, g, g, elem_bytes=eb)
         torch.cuda.synchronize()
         ok = torch.equal(buf, ref)
         del ref
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         for r in range(5):
-            ipt.ipt_010_(buf, cnt, g, g)
+            ipt.ipt_010_(buf, cnt, g, g, elem_bytes=eb)
         e1.record(); torch.cuda.synchronize()
         ms = e0.elapsed_time(e1) / 5
         rate = round(2 * cnt * g * g * eb / (ms / 1e3) / 1e9)

@@ -1,0 +1,352 @@
+// cycle_seg.cu -- elementary transposition P(batch, A, B, s) by cycle following along
+// precomputed, equal-length cycle segments (no flag bits).
+//
+// Paper: the 100! / 0100! stages shift super-elements along the cycles of Eq. (1)
+// (Sec. 5.2).  PTTWAC lets work-items start anywhere and
+// stop at a flag set by another work-item; the paper notes that cycles alone give too
+// little and too irregular parallelism ("load imbalance"), which PTTWAC's flags
+// repair dynamically.  For small, latency-bound stages (e.g. the 52 MB configs[0]
+// matrix: one dependent global round trip per chain step, walker chains of random
+// length) the makespan is set by the LONGEST chain segment, not by bandwidth.
+//
+// B200 design (beyond the paper): the planner walks the cycles of the stage's
+// permutation once on the host (O(units), cached per shape -- like a plan) and cuts
+// every cycle into segments of at most L units, L chosen so that every segment of every
+// batch item and chunk gets its own walker (tasks <= co-resident walkers).  The kernel
+// runs all segments in two phases separated by ONE grid-wide barrier:
+//   phase 1: each walker loads the super-element (chunk) at its segment's first
+//            position x into registers;
+//   phase 2: it carries it along the segment: d = next(cur), load A[d], store the carried
+//            data into d, carry A[d] on; the last step stores into the next segment's
+//            first position WITHOUT reading it (its content was taken in phase 1).
+// Every position is read once and written once; a position is only written after it was
+// read (its own walker, program order; or the next segment's walker, phase 1 < barrier),
+// so no flags, atomics or start re-checks are needed and every walker does <= L steps.
+// Walkers are G-lane groups holding R 16-byte vectors per lane (units with S % 16 == 0
+// and 16-byte aligned data only; the flag-based cycle_global covers the rest).
+#include "ipt_internal.h"
+#include "mem_ptx.cuh"
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <tuple>
+#include <vector>
+
+namespace ipt {
+
+struct SegParams {
+    char *base;
+    uint64_t ostride, istride;   // bytes between outer / inner batch items
+    uint64_t S;                  // unit (super-element) bytes, multiple of 16
+    uint64_t A;
+    FastDiv divB, divInner, divNch, divNseg;
+    uint64_t nch;                // chunks per unit
+    uint64_t chunk;              // bytes per chunk (G * R * 16)
+    const ulonglong2 *segs;      // {first position, length} per segment
+    uint64_t nseg, tasks;        // tasks = items * nseg * nch
+    unsigned int *bar;           // grid barrier counter (zeroed before the launch)
+    int store_after_load;        // IPT_SEG_SAL (default 1)
+    uint32_t zero;               // 0 at run time, opaque to the compiler
+    int diag;                    // measurement only (results invalid): 1 no barrier, 2 no phase 2,
+                                 // 4 no phase-2 stores, 8 no phase-2 loads
+};
+
+template <int G, int R>
+__global__ void __launch_bounds__(256, 4) cycle_seg_kernel(const SegParams p) {
+    const uint64_t gtid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t w = gtid / G;
+    const uint32_t l = threadIdx.x % G;
+    const bool act = w < p.tasks;
+    uint4 D[R], Bk[R];
+#pragma unroll
+    for (int v = 0; v < R; ++v) D[v] = make_uint4(0, 0, 0, 0);
+    char *ib = nullptr;
+    uint64_t cur = 0, len = 0, off0 = 0;
+    bool valid[R];
+    if (act) {
+        uint64_t rest, ch, item, seg, to, ti;
+        fdivmod(w, p.divNch, rest, ch);          // chunk fastest: a warp's walkers cover
+        fdivmod(rest, p.divNseg, item, seg);     // adjacent chunks of one unit
+        fdivmod(item, p.divInner, to, ti);
+        ib = p.base + to * p.ostride + ti * p.istride;
+        const ulonglong2 sg = p.segs[seg];
+        cur = sg.x;
+        len = sg.y;
+        off0 = ch * p.chunk + (uint64_t)l * 16;
+#pragma unroll
+        for (int v = 0; v < R; ++v) {
+            const uint64_t off = off0 + (uint64_t)v * G * 16;
+            valid[v] = off < (ch + 1) * p.chunk && off < p.S;
+            if (valid[v]) D[v] = ld_cg<16>(ib + cur * p.S + off);
+        }
+    }
+    // phase-1 loads must have returned before this thread passes the barrier
+    uint32_t f = 0;
+#pragma unroll
+    for (int v = 0; v < R; ++v) f |= fold(D[v]);
+    if ((f & p.zero) != 0) __trap();
+    __syncthreads();
+    if (threadIdx.x == 0 && !(p.diag & 1)) {
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+        atomicAdd(p.bar, 1u);
+        uint32_t seen = 0;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(seen) : "l"(p.bar) : "memory");
+        } while (seen < gridDim.x);
+    }
+    __syncthreads();
+    if (!act || (p.diag & 2)) return;
+    for (uint64_t i = 1; i <= len; ++i) {
+        uint64_t q, r;
+        fdivmod(cur, p.divB, q, r);
+        const uint64_t d = r * p.A + q;           // Eq. (1) on units: (k mod B) * A + k / B
+        char *gd = ib + d * p.S;
+        uint32_t z = 0;
+        if (i < len && !(p.diag & 8)) {
+#pragma unroll
+            for (int v = 0; v < R; ++v)
+                if (valid[v]) Bk[v] = ld_cg<16>(gd + off0 + (uint64_t)v * G * 16);
+            // Store only after the backup has arrived (address dependency): a store racing
+            // its own line's pending fill in L2 stalls the slice (measured 2.5 vs 5.8 TB/s).
+            if (p.store_after_load) {
+                uint32_t f2 = 0;
+#pragma unroll
+                for (int v = 0; v < R; ++v) f2 |= valid[v] ? fold(Bk[v]) : 0u;
+                z = f2 & p.zero;   // runtime zero: ptxas cannot fold it (and.b32 x, 0 it can)
+            }
+        }
+        if (!(p.diag & 4)) {
+#pragma unroll
+            for (int v = 0; v < R; ++v)
+                if (valid[v]) st_cg<16>(gd + z + off0 + (uint64_t)v * G * 16, D[v]);
+        }
+        if (i < len) {
+#pragma unroll
+            for (int v = 0; v < R; ++v) D[v] = Bk[v];
+        }
+        cur = d;
+    }
+}
+
+// ------------------------------------------------------------------------ host side
+namespace {
+
+struct SegPlan {
+    bool ok = false;
+    uint64_t L = 0, nseg = 0;
+    void *dev = nullptr;   // ulonglong2[nseg], library-owned, never freed (plan cache)
+};
+
+// Walk the cycles of k -> (k mod B) * A + k / B on n = A*B units; cut each non-trivial
+// cycle into segments of <= L units with L the smallest length whose segment count fits
+// `max_seg`.  Returns false when even one segment per cycle does not fit.
+bool build_segments(uint64_t A, uint64_t B, uint64_t max_seg, std::vector<ulonglong2> &out,
+                    uint64_t &L) {
+    const uint64_t n = A * B;
+    std::vector<uint64_t> seen((n + 63) / 64, 0);
+    auto next = [A, B](uint64_t k) { return (k % B) * A + k / B; };
+    std::vector<std::pair<uint64_t, uint64_t>> cycles;   // (leader, length), length >= 2
+    uint64_t nontriv = 0;
+    for (uint64_t k = 0; k < n; ++k) {
+        if (seen[k >> 6] >> (k & 63) & 1) continue;
+        uint64_t c = k, len = 0;
+        do {
+            seen[c >> 6] |= 1ull << (c & 63);
+            c = next(c);
+            ++len;
+        } while (c != k);
+        if (len >= 2) {
+            cycles.push_back({k, len});
+            nontriv += len;
+        }
+    }
+    if (cycles.empty()) { L = 0; out.clear(); return true; }
+    if (cycles.size() > max_seg) return false;
+    uint64_t lo = 1, hi = 0;
+    for (auto &c : cycles) hi = std::max(hi, c.second);
+    auto count = [&](uint64_t len) {
+        uint64_t s = 0;
+        for (auto &c : cycles) s += (c.second + len - 1) / len;
+        return s;
+    };
+    while (lo < hi) {   // smallest L with count(L) <= max_seg
+        const uint64_t mid = lo + (hi - lo) / 2;
+        if (count(mid) <= max_seg) hi = mid; else lo = mid + 1;
+    }
+    L = lo;
+    out.clear();
+    out.reserve(count(L));
+    for (auto &c : cycles) {
+        uint64_t pos = c.first;
+        for (uint64_t done = 0; done < c.second; done += L) {
+            const uint64_t len = std::min(L, c.second - done);
+            out.push_back(make_ulonglong2(pos, len));
+            for (uint64_t j = 0; j < len; ++j) pos = next(pos);
+        }
+    }
+    (void)nontriv;
+    return true;
+}
+
+struct SegCfg {
+    int G, R;
+    uint64_t nch, chunk;
+};
+
+SegCfg seg_cfg(uint64_t S) {
+    const uint64_t nv = S / 16;
+    static const int Gs[3] = {8, 16, 32};
+    SegCfg best{32, 4, (nv + 127) / 128, 32 * 4 * 16};
+    if (nv > 128) return best;
+    uint64_t bestcap = ~0ull;
+    for (int G : Gs)
+        for (int R = 1; R <= 4; ++R) {
+            const uint64_t cap = (uint64_t)G * R;
+            if (cap >= nv && cap < bestcap) { bestcap = cap; best = SegCfg{G, R, 1, cap * 16}; }
+        }
+    return best;
+}
+
+template <int G, int R>
+void *seg_kernel_ptr() { return (void *)cycle_seg_kernel<G, R>; }
+
+void *seg_kernel(int G, int R) {
+#define IPT_SEG_K(g, r) if (G == g && R == r) return seg_kernel_ptr<g, r>();
+    IPT_SEG_K(8, 1) IPT_SEG_K(8, 2) IPT_SEG_K(8, 3) IPT_SEG_K(8, 4)
+    IPT_SEG_K(16, 1) IPT_SEG_K(16, 2) IPT_SEG_K(16, 3) IPT_SEG_K(16, 4)
+    IPT_SEG_K(32, 1) IPT_SEG_K(32, 2) IPT_SEG_K(32, 3) IPT_SEG_K(32, 4)
+#undef IPT_SEG_K
+    return nullptr;
+}
+
+int seg_blocks_per_sm(void *k) {
+    static std::mutex mu;
+    static std::map<void *, int> cache;
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = cache.find(k);
+    if (it != cache.end()) return it->second;
+    int n = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k, 256, 0) != cudaSuccess) {
+        cudaGetLastError();
+        n = 0;
+    }
+    cache[k] = n;
+    return n;
+}
+
+std::mutex g_seg_mu;
+std::map<std::tuple<int, uint64_t, uint64_t, uint64_t>, std::shared_ptr<SegPlan>> g_seg_cache;
+
+std::shared_ptr<SegPlan> seg_plan(int device, uint64_t A, uint64_t B, uint64_t max_seg) {
+    const auto key = std::make_tuple(device, A, B, max_seg);
+    {
+        std::lock_guard<std::mutex> lk(g_seg_mu);
+        auto it = g_seg_cache.find(key);
+        if (it != g_seg_cache.end()) return it->second;
+    }
+    auto sp = std::make_shared<SegPlan>();
+    std::vector<ulonglong2> segs;
+    uint64_t L = 0;
+    if (build_segments(A, B, max_seg, segs, L)) {
+        sp->L = L;
+        sp->nseg = segs.size();
+        sp->ok = true;
+        if (!segs.empty()) {
+            if (cudaMalloc(&sp->dev, segs.size() * sizeof(ulonglong2)) != cudaSuccess ||
+                cudaMemcpy(sp->dev, segs.data(), segs.size() * sizeof(ulonglong2),
+                           cudaMemcpyHostToDevice) != cudaSuccess) {
+                cudaGetLastError();
+                sp->ok = false;
+            }
+        }
+    }
+    std::lock_guard<std::mutex> lk(g_seg_mu);
+    g_seg_cache[key] = sp;
+    return sp;
+}
+
+}  // namespace
+
+// Walkers a launch can keep co-resident for a stage with S-byte units (0: not applicable).
+uint64_t cycle_seg_walkers(int64_t S_bytes, int device) {
+    if (S_bytes % 16) return 0;
+    const SegCfg c = seg_cfg((uint64_t)S_bytes);
+    void *k = seg_kernel(c.G, c.R);
+    const int per_sm = device >= 0 ? seg_blocks_per_sm(k) : 4;
+    return (uint64_t)dev_props(device).sms * per_sm * 256 / c.G;
+}
+
+bool cycle_seg_applicable(const StageDesc &d) {
+    const uint64_t S = (uint64_t)(d.s * d.eb);
+    if (S % 16 || ((uintptr_t)d.base & 15)) return false;
+    if (d.outer > 1 && (d.ostride & 15)) return false;
+    return true;
+}
+
+size_t cycle_seg_ws_bytes() { return 256; }
+
+// Returns cudaErrorNotSupported when the stage does not fit one round of walkers (the
+// caller then uses the flag-based cycle_global).
+cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int device) {
+    if (!cycle_seg_applicable(d)) return cudaErrorNotSupported;
+    const uint64_t S = (uint64_t)(d.s * d.eb);
+    const SegCfg c = seg_cfg(S);
+    void *k = seg_kernel(c.G, c.R);
+    const int per_sm = seg_blocks_per_sm(k);
+    if (per_sm < 1) return cudaErrorNotSupported;
+    const uint64_t items = (uint64_t)(d.outer * d.inner);
+    const uint64_t walkers = (uint64_t)dev_props(device).sms * per_sm * 256 / c.G;
+    const uint64_t per_item = walkers / (items * c.nch);
+    if (per_item < 1) return cudaErrorNotSupported;
+    auto sp = seg_plan(device, (uint64_t)d.A, (uint64_t)d.B, per_item);
+    if (!sp->ok) return cudaErrorNotSupported;
+    if (sp->nseg == 0) return cudaSuccess;   // identity permutation
+    SegParams p{};
+    p.base = d.base;
+    p.ostride = (uint64_t)d.ostride;
+    p.istride = (uint64_t)(d.A * d.B) * S;
+    p.S = S;
+    p.A = (uint64_t)d.A;
+    p.divB = make_fastdiv((uint64_t)d.B);
+    p.divInner = make_fastdiv((uint64_t)d.inner);
+    p.divNch = make_fastdiv(c.nch);
+    p.divNseg = make_fastdiv(sp->nseg);
+    p.nch = c.nch;
+    p.chunk = c.chunk;
+    p.segs = (const ulonglong2 *)sp->dev;
+    p.nseg = sp->nseg;
+    p.tasks = items * sp->nseg * c.nch;
+    p.bar = (unsigned int *)ws;
+    p.store_after_load = (int)env_int("IPT_SEG_SAL", 1);
+    p.zero = 0;
+    p.diag = (int)env_int("IPT_SEG_DIAG", 0);
+    cudaError_t e = cudaMemsetAsync(ws, 0, sizeof(unsigned int), st);
+    if (e != cudaSuccess) return e;
+    const uint64_t blocks_needed = (p.tasks * c.G + 255) / 256;
+    const unsigned grid = (unsigned)std::min<uint64_t>(blocks_needed, (uint64_t)dev_props(device).sms * per_sm);
+    if (env_int("IPT_DEBUG", 0))
+        fprintf(stderr, "[ipt] cycle_seg A=%lld B=%lld S=%llu G=%d R=%d nch=%llu L=%llu nseg=%llu tasks=%llu grid=%u\n",
+                (long long)d.A, (long long)d.B, (unsigned long long)S, c.G, c.R,
+                (unsigned long long)c.nch, (unsigned long long)sp->L, (unsigned long long)sp->nseg,
+                (unsigned long long)p.tasks, grid);
+    void *args[] = {&p};
+    e = cudaLaunchCooperativeKernel(k, dim3(grid), dim3(256), args, 0, st);
+    note_launch();
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+// Planner estimate of the segment length L (units per walker) without walking cycles.
+uint64_t cycle_seg_est_len(int64_t units_per_item, int64_t items, int64_t S_bytes, int device) {
+    const uint64_t w = cycle_seg_walkers(S_bytes, device);
+    if (!w) return 0;
+    const SegCfg c = seg_cfg((uint64_t)S_bytes);
+    const uint64_t per_item = w / ((uint64_t)items * c.nch);
+    if (per_item < 1) return 0;
+    return ((uint64_t)units_per_item + per_item - 1) / per_item;
+}
+
+}  // namespace ipt

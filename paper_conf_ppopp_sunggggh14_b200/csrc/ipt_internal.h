@@ -83,6 +83,14 @@ struct StageDesc {
 size_t cycle_ws_bytes(const StageDesc &d);
 cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, int device);
 
+// Segmented cycle following (cycle_seg.cu): equal-length segments of the cycles computed
+// on the host (cached per shape), one grid barrier, no flags.  Needs S*eb % 16 == 0 and
+// 16-byte aligned data; uses the first 4 bytes of `ws` (>= 256 B) as barrier counter.
+// Returns cudaErrorNotSupported when not applicable (caller falls back to flags).
+cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int device);
+uint64_t cycle_seg_walkers(int64_t S_bytes, int device);
+uint64_t cycle_seg_est_len(int64_t units_per_item, int64_t items, int64_t S_bytes, int device);
+
 // Whole-tile on-chip transposition (BS kernel, Fig. 1): s must be 1
 // and an A x B tile must fit in shared memory (tile_onchip_fits()).
 bool tile_onchip_fits(int64_t A, int64_t B, int eb, int device);

@@ -59,7 +59,11 @@ def _env_clean(monkeypatch):
 
 # -------------------------------------------------------------- elementary: 100! / 0100!
 @pytest.mark.parametrize("eb", [4, 8])
-def test_ipt_100_random_shapes(eb):
+@pytest.mark.parametrize("seg", ["0", "1", "2"])
+def test_ipt_100_random_shapes(monkeypatch, eb, seg):
+    """Cycle following of super-elements: flag-based PTTWAC (IPT_CYC_SEG=0), the default
+    choice, and precomputed cycle segments wherever applicable (2)."""
+    monkeypatch.setenv("IPT_CYC_SEG", seg)
     rnd = random.Random(100 + eb)
     for _ in range(60):
         batch = rnd.choice([1, 1, 2, 3, 5])
@@ -898,3 +902,28 @@ def test_square_swap_strided_batch_tma(monkeypatch):
         blk = src[k * stride:k * stride + M * M].copy()
         assert np.array_equal(got[k * stride:k * stride + M * M], oracle.transpose_inplace(blk, M, M)), k
         assert np.array_equal(got[k * stride + M * M:(k + 1) * stride], src[k * stride + M * M:(k + 1) * stride])
+
+
+@pytest.mark.parametrize("M,N,m,n", [(1800, 7200, 1800, 180), (7200, 1800, 144, 1800),
+                                     (1800, 7200, 1800, 1800), (360, 1000, 8, 1000),
+                                     (4096, 3000, 128, 120)])
+def test_cycle_seg_full_plans(monkeypatch, M, N, m, n):
+    """Segmented cycle following inside full 2/3-stage plans (configs[0] shapes) vs the
+    oracle; and the batched form (items x segments x chunks walkers)."""
+    monkeypatch.setenv("IPT_CYC_SEG", "2")
+    p = ipt.plan(M, N, 4, 0, m=m, n=n)
+    a = seeded.matrix_np(M, N, 4)
+    t = to_dev(a, 4)
+    ipt.transpose_(t, M, N, plan_=p)
+    assert np.array_equal(to_np(t, 4), oracle.transpose_inplace(a.copy(), M, N)), (M, N, m, n)
+
+
+def test_cycle_seg_batched_and_chunked(monkeypatch):
+    """Several items and super-elements larger than one walker (chunks), 8/16-byte units."""
+    monkeypatch.setenv("IPT_CYC_SEG", "2")
+    for (batch, A, B, s, eb) in [(3, 40, 56, 600, 4), (5, 17, 31, 64, 8), (2, 100, 3, 2, 16),
+                                 (7, 64, 64, 32, 4), (1, 997, 13, 4, 4)]:
+        a = gen(batch * A * B * s, eb)
+        t = to_dev(a, eb)
+        ipt.ipt_100_(t, batch, A, B, s, elem_bytes=eb)
+        assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, s, eb)), (batch, A, B, s, eb)

@@ -76,6 +76,7 @@ struct CycParams {
     uint32_t zero;      // 0 at run time, opaque to the compiler (address-dependency knob)
     unsigned long long *stats;  // optional diagnostics (IPT_CYC_STATS=1): round counts
     int fastloop;       // steady-state chain loop (IPT_CYC_FASTLOOP, default on)
+    int sal;            // chain stores wait for the target's backup load (IPT_CYC_SAL)
 };
 
 enum : int { M_FETCH = 0, M_SCAN = 1, M_START = 2, M_CHAIN = 3, M_REFRESH = 4, M_DONE = 5 };
@@ -151,6 +152,15 @@ cycle_global_kernel(const CycParams p) {
                 old = __shfl_sync(FULL, old, g0);
                 __syncwarp();
                 if (!(old & bit)) {
+                    if (p.sal && !back_home) {   // store after the backup arrived (cycle_seg.cu)
+                        uint32_t acc = 0;
+#pragma unroll
+                        for (int r = 0; r < R; ++r) {
+                            const int v = gl + r * G;
+                            if (v < nv) acc |= fold(in[r]);
+                        }
+                        addr += (acc & p.zero);
+                    }
 #pragma unroll
                     for (int r = 0; r < R; ++r) {
                         const int v = gl + r * G;
@@ -326,6 +336,15 @@ cycle_global_kernel(const CycParams p) {
             }
         } else if (mode == M_CHAIN) {
             if (!(old & bit)) {
+                if (p.sal && !back_home) {
+                    uint32_t acc = 0;
+#pragma unroll
+                    for (int r = 0; r < R; ++r) {
+                        const int v = gl + r * G;
+                        if (v < nv) acc |= fold(in[r]);
+                    }
+                    addr += (acc & p.zero);
+                }
 #pragma unroll
                 for (int r = 0; r < R; ++r) {
                     const int v = gl + r * G;
@@ -766,6 +785,7 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
     p.fence = (int)env_int("IPT_CYC_FENCE", 1);
     p.zero = 0;
     p.fastloop = (int)env_int("IPT_CYC_FASTLOOP", 1);
+    p.sal = (int)env_int("IPT_CYC_SAL", 0);
     p.stats = env_int("IPT_CYC_STATS", 0) ? (unsigned long long *)ws + 8 : nullptr;
     cudaError_t e = cudaMemsetAsync(ws, 0, 256 + p.nwords * 4, st);
     if (e != cudaSuccess) return e;

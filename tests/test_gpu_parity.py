@@ -774,7 +774,7 @@ SQ_SIDES = [2, 3, 7, 15, 16, 17, 63, 64, 65, 100, 127, 128, 129, 255, 256, 257, 
 
 
 @pytest.mark.parametrize("eb", [1, 2, 4, 8, 16])
-@pytest.mark.parametrize("path", ["auto", "tma", "vec", "elem", "tb512"])
+@pytest.mark.parametrize("path", ["auto", "tma", "vec", "elem", "tb512", "tb512nt512"])
 def test_square_swap_sides(monkeypatch, eb, path):
     """ipt_010 on square items through the swap kernel (TMA ring by default, register
     staged, element path): every side spans ragged block edges (g not a multiple of the
@@ -783,9 +783,11 @@ def test_square_swap_sides(monkeypatch, eb, path):
     monkeypatch.setenv("IPT_SQ_FORCE", "1")
     if path == "elem":
         monkeypatch.setenv("IPT_SQ_ELEM", "1")
-    if path == "tb512":
+    if path.startswith("tb512"):
         monkeypatch.setenv("IPT_SQ_TB", "512")
-    if path in ("vec", "tb512"):
+    if path == "tb512nt512":
+        monkeypatch.setenv("IPT_SQ_NT", "512")
+    if path in ("vec", "tb512", "tb512nt512"):
         monkeypatch.setenv("IPT_SQ_TMA", "0")
     if path == "tma":
         monkeypatch.setenv("IPT_SQ_TMA", "1")

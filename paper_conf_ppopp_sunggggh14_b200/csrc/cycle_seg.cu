@@ -241,6 +241,11 @@ int seg_blocks_per_sm(void *k) {
 std::mutex g_seg_mu;
 std::map<std::tuple<int, uint64_t, uint64_t, uint64_t>, std::shared_ptr<SegPlan>> g_seg_cache;
 
+bool seg_plan_cached(int device, uint64_t A, uint64_t B, uint64_t max_seg) {
+    std::lock_guard<std::mutex> lk(g_seg_mu);
+    return g_seg_cache.count(std::make_tuple(device, A, B, max_seg)) != 0;
+}
+
 std::shared_ptr<SegPlan> seg_plan(int device, uint64_t A, uint64_t B, uint64_t max_seg) {
     const auto key = std::make_tuple(device, A, B, max_seg);
     {
@@ -302,6 +307,12 @@ cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int 
     const uint64_t walkers = (uint64_t)dev_props(device).sms * per_sm * 256 / c.G;
     const uint64_t per_item = walkers / (items * c.nch);
     if (per_item < 1) return cudaErrorNotSupported;
+    // building a segment plan allocates and copies synchronously: not during stream capture
+    // (a captured call uses an already cached plan, else the flag kernel)
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(st, &cap) != cudaSuccess) { cudaGetLastError(); cap = cudaStreamCaptureStatusActive; }
+    if (cap != cudaStreamCaptureStatusNone && !seg_plan_cached(device, (uint64_t)d.A, (uint64_t)d.B, per_item))
+        return cudaErrorNotSupported;
     auto sp = seg_plan(device, (uint64_t)d.A, (uint64_t)d.B, per_item);
     if (!sp->ok) return cudaErrorNotSupported;
     if (sp->nseg == 0) return cudaSuccess;   // identity permutation

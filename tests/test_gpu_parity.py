@@ -929,3 +929,23 @@ def test_cycle_seg_batched_and_chunked(monkeypatch):
         t = to_dev(a, eb)
         ipt.ipt_100_(t, batch, A, B, s, elem_bytes=eb)
         assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, s, eb)), (batch, A, B, s, eb)
+
+
+def test_graph_capture_of_a_plan(monkeypatch):
+    """A full transposition captured into a CUDA graph and replayed (segment plans are
+    built outside capture; a first use inside capture falls back to the flag kernel)."""
+    M, N = 1800, 7200
+    a = seeded.matrix_np(M, N, 4)
+    t = to_dev(a, 4)
+    p1, p2 = ipt.plan(M, N, 4, 0), ipt.plan(N, M, 4, 0)
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(s):
+        ipt.transpose_(t, M, N, plan_=p1, stream=s)      # warm-up: builds cached state
+        ipt.transpose_(t, N, M, plan_=p2, stream=s)
+    torch.cuda.synchronize()
+    with torch.cuda.graph(g, stream=s):
+        ipt.transpose_(t, M, N, plan_=p1, stream=s)
+    g.replay()
+    torch.cuda.synchronize()
+    assert np.array_equal(to_np(t, 4), oracle.transpose_inplace(a.copy(), M, N))

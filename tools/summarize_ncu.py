@@ -24,7 +24,7 @@ NCU = "/usr/local/cuda/bin/ncu"
 def kind(name: str):
     """Kernel family as bench.py names it: cycle_global, or tile_onchip for every tile-stage
     kernel (tile_onchip_*, tile_group_db, tile_group_generic, tile_generic_cluster)."""
-    if "cycle_global" in name or "cycle_ua" in name:
+    if "cycle_global" in name or "cycle_ua" in name or "cycle_seg" in name:
         return "cycle_global"
     if "tile_" in name:
         return "tile_onchip"

@@ -188,14 +188,18 @@ size_t ipt_stage_workspace_bytes(int64_t batch, int64_t A, int64_t B, int64_t s,
                                  int elem_bytes);
 
 /* 100! (SoA -> ASTA, Sec. 5.2): batch x [A x B x s] -> batch x [B x A x s] by
- * cycle following of s-element super-elements with one global flag bit each. */
+ * cycle following of s-element super-elements with one global flag bit each (PTTWAC);
+ * small stages of 16-byte-multiple super-elements instead follow equal-length cycle
+ * segments precomputed on the host on the first call for a shape (cached; the first
+ * call then synchronises with the device once), with no flags. */
 ipt_status ipt_100(void *d_ptr, int64_t batch, int64_t A, int64_t B, int64_t s,
                    int elem_bytes, void *d_workspace, size_t ws_bytes, void *stream);
 
 /* 010! (AoS -> ASTA, Sec. 5.1): batch x [A x B] -> batch x [B x A] (tile-local
  * transposes; on-chip when a tile fits the shared memory of one CTA, a cluster or a
- * co-resident group of CTAs (up to ~16 MB of 16-byte-vectorisable tiles), else cycle
- * following).  A given workspace must hold ipt_stage_workspace_bytes(batch, A, B, 1). */
+ * co-resident group of CTAs (up to ~16 MB of 16-byte-vectorisable tiles), square tiles
+ * (A == B, any size) by symmetric block-pair swaps, else cycle following).  A
+ * given workspace must hold ipt_stage_workspace_bytes(batch, A, B, 1). */
 ipt_status ipt_010(void *d_ptr, int64_t batch, int64_t A, int64_t B, int elem_bytes,
                    void *d_workspace, size_t ws_bytes, void *stream);
 

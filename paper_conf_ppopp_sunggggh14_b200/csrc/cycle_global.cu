@@ -709,16 +709,12 @@ size_t cycle_ws_bytes(const StageDesc &d) {
 }
 
 cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, int device) {
-    // Segmented cycle following (cycle_seg.cu): precomputed equal-length segments, no flags.
-    // IPT_CYC_SEG: 0 = never, 1 = small stages (default), 2 = whenever applicable.
-    const long segmode = env_int("IPT_CYC_SEG", 1);
-    if (segmode > 0) {
-        const uint64_t bytes = (uint64_t)d.outer * d.inner * d.A * d.B * d.s * d.eb;
-        if (segmode == 2 || bytes <= (uint64_t)env_int("IPT_CYC_SEG_MAX_MB", 256) << 20) {
-            cudaError_t e = launch_cycle_seg(d, ws, st, device);
-            if (e != cudaErrorNotSupported) return e;
-            cudaGetLastError();
-        }
+    // Segmented cycle following (cycle_seg.cu): precomputed equal-length segments, no flags,
+    // where the planner's model predicts it faster (IPT_CYC_SEG: 0 never, 2 always).
+    if (cycle_prefer_seg(d.A * d.B, d.outer * d.inner, d.s * d.eb, device)) {
+        cudaError_t e = launch_cycle_seg(d, ws, st, device);
+        if (e != cudaErrorNotSupported) return e;
+        cudaGetLastError();
     }
     Choice c = choose(d);
     const uint64_t units = (uint64_t)d.outer * d.inner * d.A * d.B * c.nchunk;

@@ -90,6 +90,7 @@ cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, i
 cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int device);
 uint64_t cycle_seg_walkers(int64_t S_bytes, int device);
 uint64_t cycle_seg_est_len(int64_t units_per_item, int64_t items, int64_t S_bytes, int device);
+bool cycle_prefer_seg(int64_t units, int64_t items, int64_t S_bytes, int device);   // plan.cpp
 
 // Whole-tile on-chip transposition (BS kernel, Fig. 1): s must be 1
 // and an A x B tile must fit in shared memory (tile_onchip_fits()).

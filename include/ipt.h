@@ -104,7 +104,9 @@ ipt_status ipt_plan_with_tiles(int64_t M, int64_t N, int64_t m, int64_t n, int e
  * N x M plan transposes it back, timed with CUDA events on `stream`; the data is
  * unchanged on return (synchronous).  The fastest plan is returned and remembered for
  * (M, N, elem_bytes, device): later ipt_plan / ipt_transpose calls use it.
- * candidates < 2 returns ipt_plan's choice without timing. */
+ * candidates < 2 returns ipt_plan's choice without timing.  Jobs <= 256 MB time at least
+ * 12 candidates; jobs smaller than L2 are timed cold (a library-owned scratch buffer of
+ * twice the L2 size, allocated on first use, is overwritten before every repetition). */
 ipt_status ipt_plan_autotune(void *d_ptr, int64_t M, int64_t N, int elem_bytes, int candidates,
                              void *stream, ipt_plan_t *out);
 

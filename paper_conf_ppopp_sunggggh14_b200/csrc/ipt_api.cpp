@@ -9,6 +9,8 @@
 // stage is a single launch regardless of `count`.
 #include "ipt_internal.h"
 
+#include <cstdio>
+
 #include <algorithm>
 #include <atomic>
 #include <cstdlib>
@@ -462,6 +464,26 @@ static ipt_status autotune_impl(void *d_ptr, int64_t count, int64_t stride, int6
     const int device = current_device();
     if (device < 0) return IPT_ERR_NO_DEVICE;
     if (M == 1 || N == 1 || candidates < 2) return ipt_plan(M, N, elem_bytes, device, out);
+    // Small jobs are latency-bound, where the cost model is least accurate and timing a
+    // candidate costs microseconds: time at least 12.  Jobs that fit in L2 are timed cold
+    // (an L2-sized scratch buffer is overwritten before every repetition, outside the
+    // events), as a single call on fresh data would run.
+    const int64_t job = mat + (count - 1) * stride;
+    if (job <= ((int64_t)256 << 20) && candidates < 12) candidates = 12;
+    void *flush = nullptr;
+    size_t flush_bytes = 0;
+    if (job < (int64_t)dev_props(device).l2_bytes) {
+        static std::mutex fmu;
+        static std::map<int, std::pair<void *, size_t>> fcache;
+        std::lock_guard<std::mutex> lk(fmu);
+        auto &f = fcache[device];
+        if (!f.first) {
+            f.second = (size_t)dev_props(device).l2_bytes * 2;
+            if (cudaMalloc(&f.first, f.second) != cudaSuccess) { cudaGetLastError(); f.first = nullptr; }
+        }
+        flush = f.first;
+        flush_bytes = f.second;
+    }
     auto cands = plan_candidates(M, N, elem_bytes, device, candidates);
     ipt_plan_t back;
     if ((s = plan_search(N, M, elem_bytes, device, &back))) return s;
@@ -476,6 +498,7 @@ static ipt_status autotune_impl(void *d_ptr, int64_t count, int64_t stride, int6
         fill_plan(M, N, cands[i].first, cands[i].second, elem_bytes, device, &p);
         float t_min = 0;
         for (int rep = 0; rep < 2; ++rep) {
+            if (flush) cudaMemsetAsync(flush, rep, flush_bytes, st);
             cudaEventRecord(e0, st);
             if ((s = run_plan((char *)d_ptr, count, stride, &p, nullptr, 0, st, nullptr))) break;
             cudaEventRecord(e1, st);
@@ -486,6 +509,10 @@ static ipt_status autotune_impl(void *d_ptr, int64_t count, int64_t stride, int6
             if (rep == 0 || ms < t_min) t_min = ms;
         }
         if (s) break;
+        if (env_int("IPT_DEBUG", 0))
+            fprintf(stderr, "[ipt] autotune %lldx%lld cand m=%lld n=%lld var=%d,%d,%d ms=%.4f\n",
+                    (long long)M, (long long)N, (long long)p.m, (long long)p.n, p.variant[0],
+                    p.variant[1], p.variant[2], t_min);
         if (i == 0 || t_min < best_ms) { best_ms = t_min; bm = cands[i].first; bn = cands[i].second; }
     }
     cudaEventDestroy(e0);

@@ -150,11 +150,12 @@ def test_plan_prefers_vector_tiles_on_large_f32():
         assert ipt.VARIANTS[p.variant[1]] == "tile_onchip"
         # 3 stages, or 2 when a whole M x n (m x N) panel fits a group of CTAs on chip
         assert p.n_stages == 3 or (p.n_stages == 2 and (p.m == M or p.n == N))
-    # panel plans (stages 2+3 fused, m = M) where the whole M x n panel fits a cluster
+    # panel plans (one of stages 1/3 elided: m = M or n = N) where the whole panel fits a
+    # group of CTAs on chip
     p = ipt.plan(7200, 18000, 4)
     assert p.n_stages >= 2 and ipt.VARIANTS[p.variant[1]] == "tile_onchip"
     if p.n_stages == 2:
-        assert p.m == 7200 and p.n * 4 >= 256
+        assert (p.m == 7200 and p.n * 4 >= 256) or (p.n == 18000 and p.m * 4 >= 256)
 
 
 def test_workspace_batch_scales():
@@ -208,3 +209,18 @@ def test_forced_square_tiles_plan_validation():
     q = ipt.plan(7200, 1800, 4, m=120, n=200)
     q.variant[1] = 4
     assert ipt.lib().ipt_workspace_bytes(ctypes.byref(q), 1) == 0   # invalid plan -> 0
+
+
+def test_cost_model_hook_ranks_single_pass_squares_and_rejects_bad_tiles():
+    """ipt__plan_cost (tooling hook): invalid tiles -> -1; for a square matrix the
+    single swap pass is predicted cheaper than any 2-stage panel plan; small jobs pay
+    per-stage overheads (a 3-stage plan costs more per byte on a small matrix than on a
+    large one with the same tiles)."""
+    L = ipt.lib()
+    f = L.ipt__plan_cost
+    f.restype = ctypes.c_double
+    f.argtypes = [ctypes.c_int64] * 4 + [ctypes.c_int, ctypes.c_int]
+    assert f(100, 100, 7, 10, 4, -1) == -1.0
+    sq = f(16384, 16384, 16384, 16384, 4, -1)
+    assert sq > 0 and all(sq < f(16384, 16384, m, 16384, 4, -1) for m in (64, 128, 256))
+    assert f(1800, 7200, 120, 120, 4, -1) > f(18000, 72000, 120, 120, 4, -1)

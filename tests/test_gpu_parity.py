@@ -949,3 +949,30 @@ def test_graph_capture_of_a_plan(monkeypatch):
     g.replay()
     torch.cuda.synchronize()
     assert np.array_equal(to_np(t, 4), oracle.transpose_inplace(a.copy(), M, N))
+
+
+@pytest.mark.parametrize("M,N,eb", [(7200, 18000, 4), (18000, 7200, 4), (9998, 12288, 4),
+                                    (14803, 8192, 4), (16384, 16384, 4), (1800, 7200, 4),
+                                    (20000, 30000, 8)])
+def test_bench_launch_configuration_autotuned(M, N, eb):
+    """The bench's launch configuration: ipt_plan_autotune (4 candidates, as bench.py) runs
+    every candidate plan forward and the model plan back -- the data must come back
+    unchanged, bit for bit -- then the tuned plan (what the timed region launches, both
+    orientations) is checked on oracle samples and on every element by the definition."""
+    dt = torch.int32 if eb == 4 else torch.int64
+    t = torch.empty(M * N, dtype=dt, device="cuda")
+    seeded.fill_device_(t, M, N, eb)
+    p = ipt.plan_autotune(t, M, N, 4)
+    ref = torch.empty_like(t)
+    seeded.fill_device_(ref, M, N, eb)
+    assert torch.equal(t, ref), "autotune must leave the data unchanged"
+    del ref
+    ipt.transpose_(t, M, N, plan_=p)
+    _check_full(t, M, N, eb, nsamp=3000)
+    q = ipt.plan_autotune(t, N, M, 4)          # the reverse orientation (next bench step)
+    ipt.transpose_(t, N, M, plan_=q)
+    ref = torch.empty_like(t)
+    seeded.fill_device_(ref, M, N, eb)
+    assert torch.equal(t, ref), (p.as_dict(), q.as_dict())
+    del t, ref
+    torch.cuda.empty_cache()

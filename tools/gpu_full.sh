@@ -18,4 +18,5 @@ timeout 900 $NCU --set full --clock-control none --import-source on -k regex:cyc
 timeout 600 $NCU --set full --clock-control none --import-source on -k regex:tile_ -s 2 -c 1 -o gpurun_out/prof_tile -f python tools/prof_one.py 12800 15000 2 > gpurun_out/prof_tile.log 2>&1
 timeout 600 $NCU --set full --clock-control none --import-source on -k regex:tile_ -s 2 -c 1 -o gpurun_out/prof_tile_generic -f python tools/prof_one.py 9998 12288 2 > gpurun_out/prof_tile_generic.log 2>&1
 timeout 600 $NCU --set full --clock-control none --import-source on -k regex:square_swap -s 1 -c 1 -o gpurun_out/prof_sq -f python tools/prof_one.py 16384 16384 2 > gpurun_out/prof_sq.log 2>&1
+timeout 900 $NCU --set full --clock-control none --import-source on -k regex:cycle_seg -s 1 -c 1 -o gpurun_out/prof_seg -f python tools/prof_one.py 20000 30000 2 8 > gpurun_out/prof_seg.log 2>&1
 ls gpurun_out

@@ -100,7 +100,7 @@ WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
 
 def full(tag):
     out = [f"# {tag}: ncu --set full captures (`tools/prof_one.py 12800 15000`, 9998 12288, "
-           "16384 16384 for square_swap)", ""]
+           "16384 16384 for square_swap, 20000 30000 f64 for cycle_seg)", ""]
     for rep in sorted(f for f in os.listdir(GO) if f.startswith("prof_") and f.endswith(".ncu-rep")):
         raw = subprocess.run([NCU, "-i", os.path.join(GO, rep), "--page", "raw", "--csv"],
                              capture_output=True, text=True).stdout

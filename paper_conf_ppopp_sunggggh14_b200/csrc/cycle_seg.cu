@@ -346,6 +346,10 @@ cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int 
                 (unsigned long long)p.tasks, grid);
     void *args[] = {&p};
     e = cudaLaunchCooperativeKernel(k, dim3(grid), dim3(256), args, 0, st);
+    if (e == cudaErrorCooperativeLaunchTooLarge || e == cudaErrorNotSupported) {
+        cudaGetLastError();            // co-residency not available here: flag kernel instead
+        return cudaErrorNotSupported;  // (the counter memset above is harmless)
+    }
     note_launch();
     return e != cudaSuccess ? e : cudaGetLastError();
 }
@@ -361,3 +365,35 @@ uint64_t cycle_seg_est_len(int64_t units_per_item, int64_t items, int64_t S_byte
 }
 
 }  // namespace ipt
+
+// Test hook (host only, not part of the ABI in include/ipt.h): build the segments of the
+// A x B unit permutation for at most max_seg walkers and verify them the way the kernel
+// uses them -- every non-fixed position is read exactly once (a segment's first position
+// in phase 1, the others as backups) and written exactly once (positions 1..len of the
+// segment); fixed points are untouched.  Returns the number of segments (L in *L_out), -1
+// if the segments do not fit max_seg, -2 if the coverage check fails.
+extern "C" int64_t ipt__seg_check(uint64_t A, uint64_t B, uint64_t max_seg, uint64_t *L_out) {
+    std::vector<ulonglong2> segs;
+    uint64_t L = 0;
+    if (!ipt::build_segments(A, B, max_seg, segs, L)) return -1;
+    if (L_out) *L_out = L;
+    const uint64_t n = A * B;
+    std::vector<uint8_t> rd(n, 0), wr(n, 0);
+    auto next = [A, B](uint64_t k) { return (k % B) * A + k / B; };
+    for (const ulonglong2 &sg : segs) {
+        if (sg.y < 1 || sg.y > L || sg.x >= n) return -2;
+        uint64_t cur = sg.x;
+        ++rd[cur];
+        for (uint64_t i = 1; i <= sg.y; ++i) {
+            const uint64_t d = next(cur);
+            if (i < sg.y) ++rd[d];
+            ++wr[d];
+            cur = d;
+        }
+    }
+    for (uint64_t k = 0; k < n; ++k) {
+        const bool fixed = next(k) == k;
+        if (fixed ? (rd[k] || wr[k]) : (rd[k] != 1 || wr[k] != 1)) return -2;
+    }
+    return (int64_t)segs.size();
+}

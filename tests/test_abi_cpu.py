@@ -224,3 +224,32 @@ def test_cost_model_hook_ranks_single_pass_squares_and_rejects_bad_tiles():
     sq = f(16384, 16384, 16384, 16384, 4, -1)
     assert sq > 0 and all(sq < f(16384, 16384, m, 16384, 4, -1) for m in (64, 128, 256))
     assert f(1800, 7200, 120, 120, 4, -1) > f(18000, 72000, 120, 120, 4, -1)
+
+
+def test_cycle_segments_cover_every_position_once():
+    """Host logic of the segmented cycle stage (cycle_seg.cu): the segments built for at
+    most W walkers read and write every moved unit exactly once (fixed points untouched,
+    P:86-89 Eq. (1) on units), with L the smallest length that fits W; the cycle count
+    bounds it from below (one segment per cycle at least)."""
+    f = ipt.lib().ipt__seg_check
+    f.restype = ctypes.c_int64
+    f.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64)]
+    L = ctypes.c_uint64(0)
+    for (A, B, W) in [(5, 3, 4), (5, 3, 100), (3, 5, 2), (64, 64, 100), (64, 64, 10000),
+                      (1800, 40, 9472), (40, 1800, 9472), (97, 89, 50), (1, 7, 3), (7, 1, 3),
+                      (2, 2, 1), (360, 1000, 3000), (17, 31, 5)]:
+        nseg = f(A, B, W, ctypes.byref(L))
+        if A == 1 or B == 1:
+            assert nseg == 0, (A, B)
+            continue
+        if nseg == -1:       # more cycles than walkers: the stage uses the flag kernel
+            assert (A, B, W) in [(64, 64, 100), (97, 89, 50), (17, 31, 5)] or W < 4, (A, B, W)
+            continue
+        assert 0 < nseg <= W, (A, B, W, nseg)
+        moved = A * B - sum(1 for k in range(A * B) if (k % B) * A + k // B == k)
+        assert L.value >= -(-moved // W), (A, B, W, L.value)
+    # 5 x 3 (P:113): 5 cycles, 3 of them fixed points -> 12 moved units in two cycles of 6
+    assert f(5, 3, 100, ctypes.byref(L)) == 12 and L.value == 1   # one unit per walker
+    assert f(5, 3, 4, ctypes.byref(L)) == 4 and L.value == 3      # 6 = 3 + 3, twice
+    assert f(5, 3, 2, ctypes.byref(L)) == 2 and L.value == 6      # one walker per cycle
+    assert f(5, 3, 1, ctypes.byref(L)) == -1                      # 2 cycles > 1 walker

@@ -241,7 +241,7 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--queues", type=int, default=4)
     ap.add_argument("--e2e-streams", type=int, default=4)
-    ap.add_argument("--autotune", type=int, default=4,
+    ap.add_argument("--autotune", type=int, default=8,
                     help="candidates timed by ipt_plan_autotune per shape (<2: model plan)")
     ap.add_argument("--algo", default="3stage", choices=["3stage", "4stage"],
                     help="4stage = the paper's Gustavson/Karlsson baseline (comparison only)")

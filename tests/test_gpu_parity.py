@@ -735,7 +735,8 @@ def test_group_split_concurrent_streams():
 @pytest.mark.parametrize("eb,batch,A,B", [(4, 2, 64, 9998), (4, 2, 9998, 64), (4, 2, 113, 8192),
                                           (4, 1, 14803, 32), (4, 1, 14803, 128), (8, 2, 3001, 61),
                                           (8, 2, 61, 3001), (4, 3, 301, 257), (4, 2, 7, 40001),
-                                          (4, 3, 1999, 31), (8, 1, 2999, 257)])
+                                          (4, 3, 1999, 31), (8, 1, 2999, 257), (4, 2, 9998, 192),
+                                          (4, 1, 14803, 256), (8, 2, 4999, 96), (4, 3, 1001, 48)])
 def test_ipt_010_group_split_element_path(eb, batch, A, B):
     """Element-path tiles (sides not multiples of 16/elem) over a CTA group: row pieces
     fetched at their global 16-byte phase and realigned in registers on write-out."""

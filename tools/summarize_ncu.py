@@ -95,7 +95,10 @@ WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "launch__block_size", "lts__t_requests_op_atom.sum",
         "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
         "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_st.sum",
-        "smsp__inst_executed.sum"]
+        "smsp__inst_executed.sum",
+        "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum",
+        "l1tex__t_sectors_pipe_lsu_mem_global_op_st.sum", "l1tex__t_requests_pipe_lsu_mem_global_op_st.sum",
+        "lts__t_sectors_op_atom.sum", "lts__t_sectors_op_red.sum"]
 
 
 def full(tag):
@@ -118,6 +121,16 @@ def full(tag):
             for w in WANT:
                 if w in d:
                     out.append(f"| {w} | {d[w]} | {u.get(w, '')} |")
+            def num(k):
+                try:
+                    return float(d.get(k, "").replace(",", ""))
+                except ValueError:
+                    return None
+            for op in ("ld", "st"):
+                sec = num(f"l1tex__t_sectors_pipe_lsu_mem_global_op_{op}.sum")
+                req = num(f"l1tex__t_requests_pipe_lsu_mem_global_op_{op}.sum")
+                if sec and req:
+                    out.append(f"| global {op} sectors / request (LSU; TMA copies not counted) | {sec / req:.2f} | |")
             stalls = sorted(((float(d[h].replace(',', '') or 0), h) for h in hdr
                              if h.startswith("smsp__pcsamp_warps_issue_stalled_") and not h.endswith("not_issued")
                              and re.match(r"^[0-9.,]+$", d[h] or "x")), reverse=True)[:6]

@@ -201,7 +201,19 @@ SegCfg seg_cfg(uint64_t S) {
     const uint64_t nv = S / 16;
     static const int Gs[3] = {8, 16, 32};
     SegCfg best{32, 4, (nv + 127) / 128, 32 * 4 * 16};
-    if (nv > 128) return best;
+    if (nv > 128) {
+        if (env_int("IPT_CYC_CHUNK256", 2) == 1) {
+            // balanced chunks on 256-byte boundaries (16 vectors), at most 2 KB each; the
+            // default is greedy 2 KB chunks (equal or faster, tools/seg_sweep.py)
+            uint64_t cv = (nv + best.nch - 1) / best.nch;
+            cv = (cv + 15) / 16 * 16;
+            if (cv > 128) cv = 128;
+            best.nch = (nv + cv - 1) / cv;
+            best.R = (int)((cv + 31) / 32);
+            best.chunk = cv * 16;
+        }
+        return best;
+    }
     uint64_t bestcap = ~0ull;
     for (int G : Gs)
         for (int R = 1; R <= 4; ++R) {

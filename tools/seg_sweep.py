@@ -2,7 +2,7 @@
 flag kernel (IPT_CYC_SEG=0) and the segmented kernel (IPT_CYC_SEG=2); prints TB/s."""
 import json, os, subprocess, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-SIZES = [64, 128, 192, 256, 320, 384, 512, 640, 768, 960, 1024, 1536, 2000, 2048, 3200, 4096]
+SIZES = json.loads(os.environ.get("SIZES", "[64, 128, 192, 256, 320, 384, 512, 640, 768, 960, 1024, 1536, 2000, 2048, 3200, 4096]"))
 if os.environ.get("_CHILD"):
     import torch
     import paper_conf_ppopp_sunggggh14_b200 as ipt
@@ -35,7 +35,9 @@ if os.environ.get("_CHILD"):
         res[S] = round(2 * n * 4 / (ms / 1e3) / 1e12, 2) if ok else "WRONG"
     print(json.dumps(res), flush=True)
 else:
+    extra = json.loads(os.environ.get("VARIANTS", "[{}]"))
     for mode in ["0", "2"]:
-        env = dict(os.environ, _CHILD="1", IPT_CYC_SEG=mode, IPT_CYC_SEG_MAX_MB="100000")
-        out = subprocess.run([sys.executable, __file__], env=env, capture_output=True, text=True)
-        print("IPT_CYC_SEG=" + mode, out.stdout.strip(), out.stderr.strip()[-400:] if out.returncode else "", flush=True)
+        for v in extra:
+            env = dict(os.environ, _CHILD="1", IPT_CYC_SEG=mode, **{k: str(x) for k, x in v.items()})
+            out = subprocess.run([sys.executable, __file__], env=env, capture_output=True, text=True)
+            print("IPT_CYC_SEG=" + mode, json.dumps(v), out.stdout.strip(), out.stderr.strip()[-400:] if out.returncode else "", flush=True)

@@ -2,7 +2,7 @@
 """Benchmark of libipt's 3-stage in-place transposition on B200 (driver contract).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                    [--workload sweep|c1|c3|c4|c5]
+                    [--workload sweep|c1|c3|c4|c5|table2]
 
 Metric (BASELINE.json): in-place transpose effective GB/s = 2*M*N*elem_bytes / time
 (PAPER.md P:56), whole job (all ranks); also reported as a fraction of the measured HBM
@@ -43,6 +43,10 @@ WORKLOADS = {
     "c4": dict(name="configs[3] large 20000x30000 float64", shapes=[(20000, 30000)], eb=8),
     "c5": dict(name="configs[4] batch of 512 4096x3000 float32", shapes=[(4096, 3000)], eb=4,
                batch=512),
+    # the paper's Table 2 shapes (~12.9 M single-precision elements each; K20:
+    # 18.7-20.7 GB/s) -- a secondary line for the paper comparison, not the headline
+    "table2": dict(name="paper Table 2 shapes (P:277-282), float32", shapes=[
+        (7200, 1800), (5100, 2500), (4000, 3200), (3300, 3900), (2500, 5100), (1800, 7200)], eb=4),
 }
 
 

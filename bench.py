@@ -352,7 +352,10 @@ def main():
     torch.cuda.synchronize()
     l2_bytes = torch.cuda.get_device_properties(dev).L2_cache_size
     resident = any(M * N * eb * cnt <= l2_bytes for (_, M, N, cnt, _) in mats)
-    # 4x L2 of flush writes per step (int32 add over 512 MB) for L2-resident matrices
+    # 4x L2 of flush READS per step (int32 sum over 512 MB) for L2-resident matrices: it
+    # evicts the previous step's data (written back here, outside the step's events) and
+    # leaves L2 full of clean lines -- a write flush would leave dirty lines whose
+    # write-back then lands inside the next timed step
     flush = torch.zeros(128 << 20, dtype=torch.int32, device=dev) if resident else None
     clocks = clock_sampler(local)
     launches0 = ipt.kernel_launch_count()
@@ -378,7 +381,7 @@ def main():
         step_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                    for _ in range(args.steps)]
         for s in range(args.steps):
-            flush.add_(1)
+            flush_sum = flush.sum()
             step_ev[s][0].record()
             one_step(step_events(s))
             step_ev[s][1].record()
@@ -571,7 +574,7 @@ def main():
                        "elem_bytes": eb, "batch": wl.get("batch", 1),
                        "plans": plans_cfg,
                        "l2": ("no flush: every matrix exceeds the 126 MB L2" if not flushed else
-                              "L2 flushed before every step (512 MB read+write, outside the step's events; "
+                              "L2 flushed before every step (512 MB read, clean lines, outside the step's events; "
                               "time = sum of per-step device times)"),
                        "parallelism": f"replicas x{world}" if "batch" not in wl else f"batch shards x{world}",
                        "algo": args.algo,

@@ -249,7 +249,7 @@ def main():
                     help="candidates timed by ipt_plan_autotune per shape (<2: model plan)")
     ap.add_argument("--stage-events", default="last", choices=["all", "last", "none"],
                     help="per-stage CUDA events (roofline per-kernel times): every timed step, "
-                         "the last one (default: an event record between every stage costs "
+                         "the last two (default: an event record between every stage costs "
                          "2.7 %% on the sweep, 17 %% on 50 MB matrices), or none")
     ap.add_argument("--algo", default="3stage", choices=["3stage", "4stage"],
                     help="4stage = the paper's Gustavson/Karlsson baseline (comparison only)")
@@ -363,10 +363,10 @@ def main():
     torch.cuda.nvtx.range_push("timed")       # ncu --nvtx --nvtx-include "timed/"
     def step_events(s):
         """Per-stage events of step s (cudaEventRecord between the stages of every matrix):
-        on every step, only the last one, or none (--stage-events)."""
+        on every step, only the last two (both orientations), or none (--stage-events)."""
         if args.algo != "3stage" or args.stage_events == "none":
             return None
-        if args.stage_events == "last" and s != args.steps - 1:
+        if args.stage_events == "last" and s < args.steps - 2:   # last two: both orientations
             return None
         return evs[s]
 

@@ -977,3 +977,17 @@ def test_bench_launch_configuration_autotuned(M, N, eb):
     assert torch.equal(t, ref), (p.as_dict(), q.as_dict())
     del t, ref
     torch.cuda.empty_cache()
+
+
+def test_full_square_f64_single_pass():
+    """A 3.2 GB square (20000^2 float64, > 2^31 bytes): the single swap pass, checked on
+    oracle samples and on every element by the definition."""
+    M = 20000
+    p = ipt.plan(M, M, 8, 0)
+    assert p.n_stages == 1 and ipt.VARIANTS[p.variant[1]] == "square_swap"
+    t = torch.empty(M * M, dtype=torch.int64, device="cuda")
+    seeded.fill_device_(t, M, M, 8)
+    ipt.transpose_(t, M, M)
+    _check_full(t, M, M, 8, nsamp=3000)
+    del t
+    torch.cuda.empty_cache()

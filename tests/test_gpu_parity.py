@@ -775,7 +775,7 @@ SQ_SIDES = [2, 3, 7, 15, 16, 17, 63, 64, 65, 100, 127, 128, 129, 255, 256, 257, 
 
 
 @pytest.mark.parametrize("eb", [1, 2, 4, 8, 16])
-@pytest.mark.parametrize("path", ["auto", "tma", "vec", "elem", "tb512", "tb512nt512"])
+@pytest.mark.parametrize("path", ["auto", "tma", "vec", "elem", "tb512", "tb512nt512", "swz", "swz512", "noswz"])
 def test_square_swap_sides(monkeypatch, eb, path):
     """ipt_010 on square items through the swap kernel (TMA ring by default, register
     staged, element path): every side spans ragged block edges (g not a multiple of the
@@ -792,6 +792,11 @@ def test_square_swap_sides(monkeypatch, eb, path):
         monkeypatch.setenv("IPT_SQ_TMA", "0")
     if path == "tma":
         monkeypatch.setenv("IPT_SQ_TMA", "1")
+    if path.startswith("swz"):
+        monkeypatch.setenv("IPT_SQ_SWZ", "1")
+        monkeypatch.setenv("IPT_SQ_TB", "512" if path == "swz512" else "256")
+    if path == "noswz":
+        monkeypatch.setenv("IPT_SQ_SWZ", "0")
     rnd = random.Random(eb * 7 + len(path))
     for g in SQ_SIDES:
         batch = rnd.choice([1, 1, 2, 3]) if g > 256 else rnd.choice([1, 2, 5, 17])

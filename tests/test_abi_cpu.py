@@ -253,3 +253,27 @@ def test_cycle_segments_cover_every_position_once():
     assert f(5, 3, 4, ctypes.byref(L)) == 4 and L.value == 3      # 6 = 3 + 3, twice
     assert f(5, 3, 2, ctypes.byref(L)) == 2 and L.value == 6      # one walker per cycle
     assert f(5, 3, 1, ctypes.byref(L)) == -1                      # 2 cycles > 1 walker
+
+
+def _build_c_example(tmp_path):
+    import shutil
+    import subprocess
+    gcc = shutil.which("gcc")
+    if not gcc or not os.path.exists("/usr/local/cuda/include/cuda_runtime.h"):
+        pytest.skip("gcc / CUDA headers not available")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    pkg = os.path.join(root, "paper_conf_ppopp_sunggggh14_b200")
+    exe = str(tmp_path / "transpose_example")
+    r = subprocess.run([gcc, "-O2", "-I", os.path.join(root, "include"), "-I", "/usr/local/cuda/include",
+                        os.path.join(root, "examples", "transpose_example.c"), "-L", pkg, "-lipt",
+                        f"-Wl,-rpath,{pkg}", "-L", "/usr/local/cuda/lib64", "-lcudart", "-o", exe],
+                       capture_output=True, text=True)
+    assert r.returncode == 0, r.stderr
+    return exe
+
+
+def test_c_example_compiles_and_links_against_the_abi(tmp_path):
+    """A plain C program (examples/transpose_example.c) builds against include/ipt.h and
+    links libipt.so: the boundary is usable without Python or torch."""
+    ipt.lib()
+    _build_c_example(tmp_path)

@@ -996,3 +996,18 @@ def test_full_square_f64_single_pass():
     _check_full(t, M, M, 8, nsamp=3000)
     del t
     torch.cuda.empty_cache()
+
+
+def test_c_example_runs(tmp_path):
+    """The C example (examples/transpose_example.c) transposes on the device through the
+    plain C ABI and verifies A^T(j, i) = A(i, j) on the host (odd and square shapes)."""
+    import subprocess
+    import importlib.util
+    spec = importlib.util.spec_from_file_location(
+        "abi_cpu", os.path.join(os.path.dirname(os.path.abspath(__file__)), "test_abi_cpu.py"))
+    mod = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mod)
+    exe = mod._build_c_example(tmp_path)
+    for (M, N) in [(1800, 7200), (997, 4093), (2048, 2048), (1, 5)]:
+        r = subprocess.run([exe, str(M), str(N)], capture_output=True, text=True, timeout=120)
+        assert r.returncode == 0 and "ok: 0 mismatches" in r.stdout, (M, N, r.stdout, r.stderr)

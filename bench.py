@@ -245,6 +245,9 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--queues", type=int, default=4)
     ap.add_argument("--e2e-streams", type=int, default=4)
+    ap.add_argument("--e2e-api", default="pipeline", choices=["pipeline", "async"],
+                    help="e2e through ipt_transpose_host_pipeline (one call per step) or "
+                         "ipt_transpose_host_async per matrix on --e2e-streams streams")
     ap.add_argument("--autotune", type=int, default=8,
                     help="candidates timed by ipt_plan_autotune per shape (<2: model plan)")
     ap.add_argument("--stage-events", default="last", choices=["all", "last", "none"],
@@ -514,6 +517,13 @@ def main():
         e2e_streams = [torch.cuda.Stream(device=dev) for _ in range(args.e2e_streams)]
 
         def e2e_step():
+            if args.e2e_api == "pipeline":   # one call: H2D / stages / D2H pipelined across matrices
+                shapes = []
+                for i, (h, M, N) in enumerate(hosts):
+                    shapes.append((N, M) if horient[i] else (M, N))
+                    horient[i] = not horient[i]
+                ipt.transpose_host_pipeline_([h for (h, _, _) in hosts], shapes)
+                return
             cur = torch.cuda.current_stream()
             for st_ in e2e_streams:
                 st_.wait_stream(cur)
@@ -542,7 +552,10 @@ def main():
         e2e = {"value": round(hb * 2 * args.e2e_steps * world / (float(ems.item()) / 1e3) / 1e9, 3),
                "unit": "GB/s", "h2d_bytes_per_step": hb, "d2h_bytes_per_step": hb,
                "steps": args.e2e_steps, "queues": args.queues, "wall_s": round(wall, 3),
-               "api": f"ipt_transpose_host_async on {len(e2e_streams)} streams (pinned host buffers, Sec. 6 queues)"}
+               "api": ("ipt_transpose_host_pipeline (one call per step: H2D of matrix i+1 and D2H of "
+                       "matrix i-1 overlap the stages of matrix i; pinned host buffers)"
+                       if args.e2e_api == "pipeline" else
+                       f"ipt_transpose_host_async on {len(e2e_streams)} streams (pinned host buffers, Sec. 6 queues)")}
         # verify one host result
         (h, M, N) = hosts[0]
         idx = torch.randint(0, M * N, (2048,))

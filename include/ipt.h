@@ -182,6 +182,19 @@ ipt_status ipt_transpose_host_async(void *h_ptr, int64_t M, int64_t N, int elem_
                                     int queues, void *d_buffer, size_t d_buffer_bytes,
                                     void *stream);
 
+/* Host-delegated transposition of `count` host matrices (h_ptrs[i]: Ms[i] x Ns[i],
+ * elem_bytes each; pinned memory for overlap) as a copy/compute pipeline across matrices
+ * (Sec. 6's overlap applied between matrices): the H2D of matrix i+1 and the D2H of matrix
+ * i-1 overlap the stages of matrix i, with two device slots, one copy-in, one compute and
+ * one copy-out stream (internal, per caller stream).  Every h_ptrs[i] is overwritten with
+ * its transpose.  d_buffer (may be NULL = internal cache) must hold 2 slots of the largest
+ * matrix (256-byte aligned) plus the stage workspace (IPT_ERR_NO_MEMORY otherwise).
+ * Asynchronous: ordered after prior work on `stream`, and `stream` continues after the
+ * last copy-out; host buffers must not be touched before that. */
+ipt_status ipt_transpose_host_pipeline(void *const *h_ptrs, const int64_t *Ms, const int64_t *Ns,
+                                       int count, int elem_bytes, void *d_buffer,
+                                       size_t d_buffer_bytes, void *stream);
+
 /* ------------------------------------------------ elementary transpositions */
 
 /* Device workspace bytes for P(batch, A, B, s) with elem_bytes elements (for s == 1 it

@@ -74,6 +74,8 @@ ABI = [
     ("ipt_transpose_4stage", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
     ("ipt_transpose_host", _int, [_vp, _i64, _i64, _int, _int, _vp, _sz, _vp]),
     ("ipt_transpose_host_async", _int, [_vp, _i64, _i64, _int, _int, _vp, _sz, _vp]),
+    ("ipt_transpose_host_pipeline", _int,
+     [ctypes.POINTER(_vp), ctypes.POINTER(_i64), ctypes.POINTER(_i64), _int, _int, _vp, _sz, _vp]),
     ("ipt_stage_workspace_bytes", _sz, [_i64, _i64, _i64, _i64, _int]),
     ("ipt_100", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
     ("ipt_010", _int, [_vp, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
@@ -279,6 +281,29 @@ def transpose_host_async_(h, M: int, N: int, queues: int = 4, stream=None,
     _check(lib().ipt_transpose_host_async(ctypes.c_void_p(h.data_ptr()), M, N, eb, queues, None, 0,
                                           _stream_ptr(stream)), "ipt_transpose_host_async")
     return h
+
+
+def transpose_host_pipeline_(hs, shapes, stream=None, elem_bytes: int | None = None):
+    """Host-delegated transposition of several host tensors (pinned for overlap) as one
+    copy/compute pipeline: hs[i] holds a shapes[i] = (M, N) matrix and is overwritten with
+    its transpose.  Asynchronous on `stream`; synchronise it before reading the tensors."""
+    if len(hs) != len(shapes):
+        raise IptError("one (M, N) per tensor")
+    if not hs:
+        return hs
+    eb = _eb(hs[0], elem_bytes)
+    for h, (M, N) in zip(hs, shapes):
+        if h.is_cuda or not h.is_contiguous():
+            raise IptError("transpose_host_pipeline_ expects contiguous host tensors")
+        if _nelem(h, eb) != M * N:
+            raise IptError(f"elements {_nelem(h, eb)} != M*N {M * N}")
+    n = len(hs)
+    ptrs = (ctypes.c_void_p * n)(*[h.data_ptr() for h in hs])
+    Ms = (ctypes.c_int64 * n)(*[M for (M, _) in shapes])
+    Ns = (ctypes.c_int64 * n)(*[N for (_, N) in shapes])
+    _check(lib().ipt_transpose_host_pipeline(ptrs, Ms, Ns, n, eb, None, 0, _stream_ptr(stream)),
+           "ipt_transpose_host_pipeline")
+    return hs
 
 
 # ----------------------------------------------------------- elementary transpositions

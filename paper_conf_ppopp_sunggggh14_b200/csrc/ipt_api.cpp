@@ -141,13 +141,13 @@ WsCache &ws_cache() {
 }
 
 // Internal buffers are cached per (device, stream, purpose): `purpose` 0 = flag workspace,
-// 1 = host-path staging buffer.  Growing a buffer synchronises `stream` first (work
+// 1 = host-path staging buffer, 2 = host pipeline buffers.  Growing a buffer synchronises `stream` first (work
 // already enqueued on it may still use the old buffer).
 ipt_status get_ws(int device, void *stream, size_t need, void **out, int purpose = 0) {
     if (need == 0) { *out = nullptr; return IPT_OK; }
     WsCache &c = ws_cache();
     std::lock_guard<std::mutex> lk(c.mu);
-    auto key = std::make_pair(device * 2 + purpose, stream);
+    auto key = std::make_pair(device * 4 + purpose, stream);
     auto it = c.bufs.find(key);
     if (it != c.bufs.end() && it->second.second >= need) {
         *out = it->second.first;
@@ -716,6 +716,116 @@ static ipt_status transpose_host_impl(void *h_ptr, int64_t M, int64_t N, int ele
     cudaEventDestroy(ev1);   // released once the recorded work completes
     for (auto d : done) cudaEventDestroy(d);
     return cuda_status(e);
+}
+
+// Host pipeline (Sec. 6 across matrices): H2D of matrix i+1 and D2H of matrix i-1 overlap
+// the stages of matrix i -- two device slots, a copy-in stream, a compute stream and a
+// copy-out stream per (device, caller stream); slot reuse waits for its D2H.
+static ipt_status pipe_streams(int device, void *caller, cudaStream_t out[3]) {
+    static std::mutex mu;
+    static std::map<std::pair<int, void *>, std::vector<cudaStream_t>> cache;
+    std::lock_guard<std::mutex> lk(mu);
+    auto &v = cache[std::make_pair(device, caller)];
+    while (v.size() < 3) {
+        cudaStream_t s;
+        if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) {
+            cudaGetLastError();
+            return IPT_ERR_CUDA;
+        }
+        v.push_back(s);
+    }
+    for (int i = 0; i < 3; ++i) out[i] = v[i];
+    return IPT_OK;
+}
+
+ipt_status ipt_transpose_host_pipeline(void *const *h_ptrs, const int64_t *Ms, const int64_t *Ns,
+                                       int count, int elem_bytes, void *d_buffer,
+                                       size_t d_buffer_bytes, void *stream) {
+    if (count < 0 || (count > 0 && (!h_ptrs || !Ms || !Ns))) return IPT_ERR_INVALID_ARG;
+    if (count == 0) return IPT_OK;
+    if (!elem_ok(elem_bytes)) return IPT_ERR_UNSUPPORTED_ELEM;
+    int64_t maxb = 0;
+    for (int i = 0; i < count; ++i) {
+        int64_t b = 0;
+        ipt_status s = check_shape(Ms[i], Ns[i], elem_bytes, &b);
+        if (s) return s;
+        if ((s = check_ptr(h_ptrs[i], elem_bytes))) return s;
+        maxb = std::max(maxb, b);
+    }
+    const int device = current_device();
+    if (device < 0) return IPT_ERR_NO_DEVICE;
+    std::vector<ipt_plan_t> plans(count);
+    size_t ws = 0;
+    for (int i = 0; i < count; ++i) {
+        if (Ms[i] == 1 || Ns[i] == 1) continue;
+        ipt_status s = ipt_plan(Ms[i], Ns[i], elem_bytes, device, &plans[i]);
+        if (s) return s;
+        ws = std::max(ws, batched_ws(&plans[i], 1));
+    }
+    const size_t slot = align256((size_t)maxb);
+    const size_t need = 2 * slot + align256(ws);
+    char *dbuf = (char *)d_buffer;
+    if (!dbuf) {
+        void *w = nullptr;
+        ipt_status s = get_ws(device, stream, need, &w, 2);
+        if (s) return s;
+        dbuf = (char *)w;
+    } else if (d_buffer_bytes < need) {
+        return IPT_ERR_NO_MEMORY;
+    }
+    char *dws = dbuf + 2 * slot;
+    cudaStream_t qs[3];
+    ipt_status s = pipe_streams(device, stream, qs);
+    if (s) return s;
+    cudaStream_t st = (cudaStream_t)stream, H = qs[0], C = qs[1], D = qs[2];
+    cudaEvent_t start, h2d[2], comp[2], d2h[2];
+    cudaEventCreateWithFlags(&start, cudaEventDisableTiming);
+    for (int k = 0; k < 2; ++k) {
+        cudaEventCreateWithFlags(&h2d[k], cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&comp[k], cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&d2h[k], cudaEventDisableTiming);
+    }
+    cudaEventRecord(start, st);               // everything follows prior work on `stream`
+    cudaStreamWaitEvent(H, start, 0);
+    cudaStreamWaitEvent(C, start, 0);
+    cudaStreamWaitEvent(D, start, 0);
+    cudaError_t e = cudaSuccess;
+    for (int i = 0; i < count && e == cudaSuccess; ++i) {
+        if (Ms[i] == 1 || Ns[i] == 1) continue;   // the layout is already its transpose
+        const int k = i & 1;
+        char *b = dbuf + k * slot;
+        const size_t bytes = (size_t)(Ms[i] * Ns[i] * elem_bytes);
+        if (i >= 2) cudaStreamWaitEvent(H, d2h[k], 0);   // slot k free again
+        e = cudaMemcpyAsync(b, h_ptrs[i], bytes, cudaMemcpyHostToDevice, H);
+        if (e != cudaSuccess) break;
+        cudaEventRecord(h2d[k], H);
+        cudaStreamWaitEvent(C, h2d[k], 0);
+        ipt_status r = run_plan(b, 1, (int64_t)bytes, &plans[i], dws, align256(ws), C, nullptr);
+        if (r) { e = cudaErrorUnknown; s = r; break; }
+        cudaEventRecord(comp[k], C);
+        cudaStreamWaitEvent(D, comp[k], 0);
+        e = cudaMemcpyAsync(h_ptrs[i], b, bytes, cudaMemcpyDeviceToHost, D);
+        if (e != cudaSuccess) break;
+        cudaEventRecord(d2h[k], D);
+    }
+    // join: `stream` continues after every copy-out
+    cudaEvent_t done;
+    cudaEventCreateWithFlags(&done, cudaEventDisableTiming);
+    cudaEventRecord(done, D);
+    cudaStreamWaitEvent(st, done, 0);
+    cudaEventRecord(done, C);                  // (re-recorded: C and H end before D anyway)
+    cudaStreamWaitEvent(st, done, 0);
+    cudaEventRecord(done, H);
+    cudaStreamWaitEvent(st, done, 0);
+    cudaEventDestroy(done);
+    cudaEventDestroy(start);
+    for (int k = 0; k < 2; ++k) {
+        cudaEventDestroy(h2d[k]);
+        cudaEventDestroy(comp[k]);
+        cudaEventDestroy(d2h[k]);
+    }
+    if (s) return s;
+    return cuda_status(e != cudaSuccess ? e : cudaGetLastError());
 }
 
 ipt_status ipt_transpose_host(void *h_ptr, int64_t M, int64_t N, int elem_bytes, int queues,

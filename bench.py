@@ -245,9 +245,10 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--queues", type=int, default=4)
     ap.add_argument("--e2e-streams", type=int, default=4)
-    ap.add_argument("--e2e-api", default="pipeline", choices=["pipeline", "async"],
-                    help="e2e through ipt_transpose_host_pipeline (one call per step) or "
-                         "ipt_transpose_host_async per matrix on --e2e-streams streams")
+    ap.add_argument("--e2e-api", default="async", choices=["pipeline", "async"],
+                    help="e2e through ipt_transpose_host_async per matrix on --e2e-streams streams "
+                         "(default: 80 GB/s) or ipt_transpose_host_pipeline, one call per step "
+                         "(76 GB/s: one copy engine per direction)")
     ap.add_argument("--autotune", type=int, default=8,
                     help="candidates timed by ipt_plan_autotune per shape (<2: model plan)")
     ap.add_argument("--stage-events", default="last", choices=["all", "last", "none"],

@@ -150,7 +150,6 @@ bool build_segments(uint64_t A, uint64_t B, uint64_t max_seg, std::vector<ulongl
     std::vector<uint64_t> seen((n + 63) / 64, 0);
     auto next = [A, B](uint64_t k) { return (k % B) * A + k / B; };
     std::vector<std::pair<uint64_t, uint64_t>> cycles;   // (leader, length), length >= 2
-    uint64_t nontriv = 0;
     for (uint64_t k = 0; k < n; ++k) {
         if (seen[k >> 6] >> (k & 63) & 1) continue;
         uint64_t c = k, len = 0;
@@ -159,10 +158,7 @@ bool build_segments(uint64_t A, uint64_t B, uint64_t max_seg, std::vector<ulongl
             c = next(c);
             ++len;
         } while (c != k);
-        if (len >= 2) {
-            cycles.push_back({k, len});
-            nontriv += len;
-        }
+        if (len >= 2) cycles.push_back({k, len});
     }
     if (cycles.empty()) { L = 0; out.clear(); return true; }
     if (cycles.size() > max_seg) return false;
@@ -188,7 +184,6 @@ bool build_segments(uint64_t A, uint64_t B, uint64_t max_seg, std::vector<ulongl
             for (uint64_t j = 0; j < len; ++j) pos = next(pos);
         }
     }
-    (void)nontriv;
     return true;
 }
 
@@ -297,9 +292,14 @@ uint64_t cycle_seg_walkers(int64_t S_bytes, int device) {
     return (uint64_t)dev_props(device).sms * per_sm * 256 / c.G;
 }
 
+// Host cycle walk bound: ~10 ns per unit, once per shape; beyond 2^26 units (~0.7 s) the
+// flag kernel is used instead.
+constexpr uint64_t kSegMaxUnits = 1ull << 26;
+
 bool cycle_seg_applicable(const StageDesc &d) {
     const uint64_t S = (uint64_t)(d.s * d.eb);
     if (S % 16 || ((uintptr_t)d.base & 15)) return false;
+    if ((uint64_t)(d.A * d.B) > kSegMaxUnits) return false;
     if (d.outer > 1 && (d.ostride & 15)) return false;
     return true;
 }
@@ -368,6 +368,7 @@ cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int 
 
 // Planner estimate of the segment length L (units per walker) without walking cycles.
 uint64_t cycle_seg_est_len(int64_t units_per_item, int64_t items, int64_t S_bytes, int device) {
+    if ((uint64_t)units_per_item > kSegMaxUnits) return 0;
     const uint64_t w = cycle_seg_walkers(S_bytes, device);
     if (!w) return 0;
     const SegCfg c = seg_cfg((uint64_t)S_bytes);

@@ -48,7 +48,8 @@ struct SegParams {
     uint64_t chunk;              // bytes per chunk (G * R * 16)
     const ulonglong2 *segs;      // {first position, length} per segment
     uint64_t nseg, tasks;        // tasks = items * nseg * nch
-    unsigned int *bar;           // grid barrier counter (zeroed before the launch)
+    unsigned int *bar;           // grid barrier counters [arrive, exit]
+    int self_reset;              // counters start at 0 and the last CTA re-zeroes them
     int store_after_load;        // IPT_SEG_SAL (default 1)
     uint32_t zero;               // 0 at run time, opaque to the compiler
     int diag;                    // measurement only (results invalid): 1 no barrier, 2 no phase 2,
@@ -97,6 +98,12 @@ __global__ void __launch_bounds__(256, 4) cycle_seg_kernel(const SegParams p) {
         do {
             asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(seen) : "l"(p.bar) : "memory");
         } while (seen < gridDim.x);
+        if (p.self_reset && atomicAdd(p.bar + 1, 1u) == gridDim.x - 1) {
+            // every CTA has left the spin: zero both counters for the next launch on this
+            // stream (stream order makes them visible to it), no memset node needed
+            atomicExch(p.bar, 0u);
+            atomicExch(p.bar + 1, 0u);
+        }
     }
     __syncthreads();
     if (!act || (p.diag & 2)) return;
@@ -248,6 +255,31 @@ int seg_blocks_per_sm(void *k) {
 std::mutex g_seg_mu;
 std::map<std::tuple<int, uint64_t, uint64_t, uint64_t>, std::shared_ptr<SegPlan>> g_seg_cache;
 
+// Self-resetting barrier counters, one zero-initialised pair per (device, stream); created
+// synchronously on first use (never inside stream capture), never freed.
+std::mutex g_ctr_mu;
+std::map<std::pair<int, cudaStream_t>, unsigned int *> g_ctr;
+
+unsigned int *seg_counters_cached(int device, cudaStream_t st) {
+    std::lock_guard<std::mutex> lk(g_ctr_mu);
+    auto it = g_ctr.find(std::make_pair(device, st));
+    return it == g_ctr.end() ? nullptr : it->second;
+}
+
+unsigned int *seg_counters(int device, cudaStream_t st) {
+    std::lock_guard<std::mutex> lk(g_ctr_mu);
+    auto key = std::make_pair(device, st);
+    auto it = g_ctr.find(key);
+    if (it != g_ctr.end()) return it->second;
+    void *p = nullptr;
+    if (cudaMalloc(&p, 256) != cudaSuccess || cudaMemset(p, 0, 256) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    g_ctr[key] = (unsigned int *)p;
+    return (unsigned int *)p;
+}
+
 bool seg_plan_cached(int device, uint64_t A, uint64_t B, uint64_t max_seg) {
     std::lock_guard<std::mutex> lk(g_seg_mu);
     return g_seg_cache.count(std::make_tuple(device, A, B, max_seg)) != 0;
@@ -343,12 +375,25 @@ cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int 
     p.segs = (const ulonglong2 *)sp->dev;
     p.nseg = sp->nseg;
     p.tasks = items * sp->nseg * c.nch;
-    p.bar = (unsigned int *)ws;
     p.store_after_load = (int)env_int("IPT_SEG_SAL", 1);
     p.zero = 0;
     p.diag = (int)env_int("IPT_SEG_DIAG", 0);
-    cudaError_t e = cudaMemsetAsync(ws, 0, sizeof(unsigned int), st);
-    if (e != cudaSuccess) return e;
+    // barrier counters: a library-owned, self-resetting pair per (device, stream) -- no memset
+    // node per launch (2 us of a ~40 us configs[0] transposition); the caller's workspace
+    // with a memset when the pair cannot be created (e.g. first use inside stream capture)
+    unsigned int *ctr = nullptr;
+    if (env_int("IPT_SEG_RESET", 1))
+        ctr = cap == cudaStreamCaptureStatusNone ? seg_counters(device, st) : seg_counters_cached(device, st);
+    cudaError_t e = cudaSuccess;
+    if (ctr) {
+        p.bar = ctr;
+        p.self_reset = 1;
+    } else {
+        p.bar = (unsigned int *)ws;
+        p.self_reset = 0;
+        e = cudaMemsetAsync(ws, 0, 2 * sizeof(unsigned int), st);
+        if (e != cudaSuccess) return e;
+    }
     const uint64_t blocks_needed = (p.tasks * c.G + 255) / 256;
     const unsigned grid = (unsigned)std::min<uint64_t>(blocks_needed, (uint64_t)dev_props(device).sms * per_sm);
     if (env_int("IPT_DEBUG", 0))

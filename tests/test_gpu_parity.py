@@ -926,9 +926,13 @@ def test_cycle_seg_full_plans(monkeypatch, M, N, m, n):
     assert np.array_equal(to_np(t, 4), oracle.transpose_inplace(a.copy(), M, N)), (M, N, m, n)
 
 
-def test_cycle_seg_batched_and_chunked(monkeypatch):
-    """Several items and super-elements larger than one walker (chunks), 8/16-byte units."""
+@pytest.mark.parametrize("reset", ["1", "0"])
+def test_cycle_seg_batched_and_chunked(monkeypatch, reset):
+    """Several items and super-elements larger than one walker (chunks), 8/16-byte units;
+    self-resetting barrier counters (reused launch after launch on one stream) or a
+    memset of the workspace counters per launch."""
     monkeypatch.setenv("IPT_CYC_SEG", "2")
+    monkeypatch.setenv("IPT_SEG_RESET", reset)
     for (batch, A, B, s, eb) in [(3, 40, 56, 600, 4), (5, 17, 31, 64, 8), (2, 100, 3, 2, 16),
                                  (7, 64, 64, 32, 4), (1, 997, 13, 4, 4)]:
         a = gen(batch * A * B * s, eb)
@@ -1034,3 +1038,27 @@ def test_transpose_host_pipeline(eb):
     torch.cuda.synchronize()
     for h, ref, sh in zip(hs, refs, shapes):
         assert np.array_equal(h.numpy().view(ref.dtype), ref), sh
+
+
+def test_cycle_seg_counters_across_streams_and_many_launches(monkeypatch):
+    """Self-resetting barrier counters: many back-to-back segmented launches on two streams
+    (one counter pair each), every result bit-exact."""
+    monkeypatch.setenv("IPT_CYC_SEG", "2")
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    cases = [(2, 40, 56, 64), (1, 180, 40, 36)]
+    ts, refs = [], []
+    for (b, A, B, s_) in cases:
+        a = gen(b * A * B * s_, 4)
+        ts.append(to_dev(a, 4))
+        refs.append(a)
+    torch.cuda.synchronize()
+    for it in range(40):
+        for k, (b, A, B, s_) in enumerate(cases):
+            with torch.cuda.stream(streams[k]):
+                if it % 2 == 0:
+                    ipt.ipt_100_(ts[k], b, A, B, s_, stream=streams[k])
+                else:
+                    ipt.ipt_100_(ts[k], b, B, A, s_, stream=streams[k])
+    torch.cuda.synchronize()
+    for k in range(2):
+        assert np.array_equal(to_np(ts[k], 4), refs[k].view(np.uint32)), k

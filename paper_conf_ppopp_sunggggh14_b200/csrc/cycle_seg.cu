@@ -272,7 +272,9 @@ unsigned int *seg_counters(int device, cudaStream_t st) {
     auto it = g_ctr.find(key);
     if (it != g_ctr.end()) return it->second;
     void *p = nullptr;
-    if (cudaMalloc(&p, 256) != cudaSuccess || cudaMemset(p, 0, 256) != cudaSuccess) {
+    // zeroed ON the stream that uses the pair (a legacy-stream cudaMemset is not ordered
+    // before work on a non-blocking stream -- found on the host pipeline's compute stream)
+    if (cudaMalloc(&p, 256) != cudaSuccess || cudaMemsetAsync(p, 0, 256, st) != cudaSuccess) {
         cudaGetLastError();
         return nullptr;
     }
@@ -300,9 +302,12 @@ std::shared_ptr<SegPlan> seg_plan(int device, uint64_t A, uint64_t B, uint64_t m
         sp->nseg = segs.size();
         sp->ok = true;
         if (!segs.empty()) {
+            // cudaMemcpy from pageable memory may return before the DMA lands, and a
+            // non-blocking stream is not ordered after it: wait for it (once per shape)
             if (cudaMalloc(&sp->dev, segs.size() * sizeof(ulonglong2)) != cudaSuccess ||
                 cudaMemcpy(sp->dev, segs.data(), segs.size() * sizeof(ulonglong2),
-                           cudaMemcpyHostToDevice) != cudaSuccess) {
+                           cudaMemcpyHostToDevice) != cudaSuccess ||
+                cudaDeviceSynchronize() != cudaSuccess) {
                 cudaGetLastError();
                 sp->ok = false;
             }

@@ -55,6 +55,8 @@ struct TileParams {
     uint32_t ralign;      // generic cluster row split: slice boundaries in multiples of this
     uint32_t gb;          // streaming kernel: V-row blocks per group (0 = automatic)
     uint32_t *gbar;       // group-split kernel: one arrival counter per group (workspace)
+    uint32_t *gexit;      // group-split kernel: per-group exit counters (self-resetting
+                          // library-owned counters; nullptr = gbar zeroed by a memset)
     int vec16;            // generic path: tiles 16-byte aligned, 16-byte loads
     int arrive_release;   // group kernels: release-ordered arrivals (default relaxed)
     uint32_t box_rows;    // tile_group_tma: rows per 2-D TMA box (divides the slice rows)
@@ -583,6 +585,16 @@ __device__ __forceinline__ void group_loop(const TileParams &p, uint32_t s0, uin
         uint32_t smid;
         asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
         tr[(kTraceIters - 1) * 4] = smid;
+    }
+    if (p.gexit && threadIdx.x == 0) {
+        // self-resetting counters: the last CTA of the group to finish (no CTA of it polls
+        // any more) zeroes the group's arrival counters and its exit counter, so the next
+        // launch on this stream starts from zero without a memset node
+        uint32_t *ex = p.gexit + gid * (kGroupCtrStride / 4);
+        if (atomicAdd(ex, 1u) == K - 1) {
+            for (uint32_t b = 0; b < p.nbuf; ++b) atomicExch(pipe.slot(b), 0u);
+            atomicExch(ex, 0u);
+        }
     }
 }
 
@@ -1385,8 +1397,30 @@ bool group_tma_setup_generic(const StageDesc &d, TileParams &p, const GroupCfg &
     return true;
 }
 
+// Library-owned group counters per (device, stream): arrivals (kTileWsBytes) then per-group
+// exit counters (kTileWsBytes), zeroed once ON that stream, re-zeroed by each launch's last
+// CTA of every group.  Not created during stream capture (create == false).
+static uint32_t *group_counters(int device, cudaStream_t st, bool create) {
+    static std::mutex mu;
+    static std::map<std::pair<int, cudaStream_t>, uint32_t *> cache;
+    std::lock_guard<std::mutex> lk(mu);
+    auto key = std::make_pair(device, st);
+    auto it = cache.find(key);
+    if (it != cache.end()) return it->second;
+    if (!create) return nullptr;
+    void *p = nullptr;
+    if (cudaMalloc(&p, 2 * kTileWsBytes) != cudaSuccess ||
+        cudaMemsetAsync(p, 0, 2 * kTileWsBytes, st) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    cache[key] = (uint32_t *)p;
+    return (uint32_t *)p;
+}
+
 // Group-split launch: groups x K CTAs, all co-resident (cooperative launch); the arrival
-// counters (workspace, kGroupCtrStride bytes apart) are zeroed on the stream first.
+// counters (kGroupCtrStride bytes apart) are library-owned and self-resetting, or the
+// call's workspace zeroed on the stream first.
 template <int EB, bool GENERIC>
 cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g, void *ws,
                             cudaStream_t st, int device) {
@@ -1403,11 +1437,24 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
     p.buf_bytes = (uint32_t)g.slice;
     p.gbar = (uint32_t *)ws;
     if ((size_t)g.groups * g.nbuf * kGroupCtrStride > kTileWsBytes) return cudaErrorInvalidValue;
+    // self-resetting counters owned by the library per (device, stream) when available
+    p.gexit = nullptr;
+    if (env_int("IPT_TILE_RESET", 1)) {
+        cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+        if (cudaStreamIsCapturing(st, &cap) != cudaSuccess) { cudaGetLastError(); cap = cudaStreamCaptureStatusActive; }
+        if (uint32_t *c = group_counters(device, st, cap == cudaStreamCaptureStatusNone)) {
+            p.gbar = c;
+            p.gexit = c + kTileWsBytes / 4;
+        }
+    }
     auto kern = GENERIC ? tile_group_generic<EB> : tile_group_db<EB>;
     CUtensorMap tmap;
     const bool tma = GENERIC ? group_tma_setup_generic<EB>(d, p, g, &tmap) : group_tma_setup<EB>(d, p, g, &tmap);
-    cudaError_t e = cudaMemsetAsync(ws, 0, (size_t)g.groups * g.nbuf * kGroupCtrStride, st);
-    if (e != cudaSuccess) return e;
+    cudaError_t e = cudaSuccess;
+    if (!p.gexit) {
+        e = cudaMemsetAsync(ws, 0, (size_t)g.groups * g.nbuf * kGroupCtrStride, st);
+        if (e != cudaSuccess) return e;
+    }
     auto set_smem = [&](const void *k) {   // dynamic + static shared memory within the opt-in maximum
         static std::mutex mu;
         static std::map<std::pair<const void *, int>, bool> done;

@@ -66,6 +66,18 @@ def test_validation_before_device():
     assert L.ipt_transpose_batched(ctypes.c_void_p(256), 2, 4, 4, 4, 4, null) == 1  # stride too small
     p = ipt.Plan()
     assert L.ipt_plan_with_tiles(12, 10, 5, 5, 4, -1, ctypes.byref(p)) == 1   # 5 does not divide 12
+    # host pipeline: arguments checked before the device is touched
+    f = L.ipt_transpose_host_pipeline
+    P = (ctypes.c_void_p * 2)(256, 512)
+    Ms, Ns = (ctypes.c_int64 * 2)(4, 8), (ctypes.c_int64 * 2)(4, 8)
+    assert f(P, Ms, Ns, 0, 4, null, 0, null) == 0                             # nothing to do
+    assert f(P, Ms, Ns, -1, 4, null, 0, null) == 1                            # count < 0
+    assert f(None, Ms, Ns, 2, 4, null, 0, null) == 1                          # NULL arrays
+    assert f(P, Ms, Ns, 2, 3, null, 0, null) == 2                             # elem 3
+    bad = (ctypes.c_int64 * 2)(4, 0)
+    assert f(P, bad, Ns, 2, 4, null, 0, null) == 1                            # M < 1
+    Pm = (ctypes.c_void_p * 2)(256, 514)
+    assert f(Pm, Ms, Ns, 2, 4, null, 0, null) == 3                            # misaligned host pointer
 
 
 def test_fastdiv_exact():

@@ -690,6 +690,69 @@ __global__ void __launch_bounds__(512, 1) tile_group_tma(const TileParams p, con
         });
 }
 
+// --------------------------------- group-split element path with TMA slices (aligned rows)
+// Element-path tiles whose INPUT rows are 16-byte aligned (n * elem % 16 == 0, row split)
+// while the output rows are not (m % (16/elem) != 0, e.g. 9998 x 192 or 14803 x 128
+// panels): slices are fetched as tile_group_tma does (2-D TMA boxes into column panels of q
+// odd vectors; boxes may cover the next tile's first rows -- read, never used), the
+// write-out reads one aligned LDS.128 per lane and 4 columns (no realignment) and stores one
+// element per lane and output row (32 consecutive output elements per warp store).
+template <int EB>
+__global__ void __launch_bounds__(512, 1) tile_group_tma_elem(const TileParams p, const __grid_constant__ CUtensorMap tmap) {
+    constexpr uint32_t V = 16 / EB;
+    using E = typename Elem<EB>::T;
+    extern __shared__ __align__(128) unsigned char smem[];
+    const uint32_t s0 = smem_u32(smem);
+    const uint32_t K = p.K, rank = blockIdx.x % K;
+    const uint32_t mvc = (p.m + V - 1) / V;                    // V-row blocks (last partial)
+    const uint32_t b0 = (uint32_t)((uint64_t)rank * mvc / K), b1 = (uint32_t)((uint64_t)(rank + 1) * mvc / K);
+    const uint32_t r0 = b0 * V, r1 = min(b1 * V, p.m);
+    const uint32_t rows = r1 > r0 ? r1 - r0 : 0;
+    const uint32_t frows = ((mvc + K - 1) / K) * V;            // rows fetched per slice
+    const uint32_t q = p.q, nvr = p.n / V;
+    constexpr uint32_t CH = 8;                                   // vector columns per task
+    const uint32_t nrb = (rows + 31) / 32, nch = (nvr + CH - 1) / CH, ntask = nrb * nch;
+    const FastDiv32 divrb = make_fastdiv32_dev(nrb ? nrb : 1), divq = make_fastdiv32_dev(q);
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+    const uint64_t mEB = (uint64_t)p.m * EB;
+    __shared__ __align__(8) uint64_t mbar[kGroupMaxBuf];
+    group_loop(p, s0, mbar,
+        [&](const char *g, uint32_t sb) {
+            if (threadIdx.x == 0) {
+                const uint64_t row0 = (uint64_t)(g - p.base) / ((uint64_t)p.n * EB) + r0;
+                uint64_t *bar = &mbar[(sb - s0) / p.buf_bytes];
+                mbar_expect_tx(bar, p.npan * frows * q * 16);
+                const uint32_t sbar = smem_u32(bar);
+                for (uint32_t pn = 0; pn < p.npan; ++pn)
+                    for (uint32_t r = 0; r < frows; r += p.box_rows)
+                        tma_load_2d(sb + pn * p.pstride + r * q * 16, &tmap, (int32_t)(pn * q * V),
+                                    (int32_t)(row0 + r), sbar);
+            }
+        },
+        [&](char *g, uint32_t sb, auto probe) {
+            for (uint32_t task = warp; task < ntask; task += nw) {
+                probe();
+                uint32_t ch, rb;
+                fdivmod32(task, divrb, ch, rb);
+                const uint32_t i = rb * 32 + lane;
+                if (i >= rows) continue;
+                char *out = g + ((uint64_t)(ch * CH) * V * p.m + r0 + i) * EB;
+#pragma unroll 2
+                for (uint32_t cbl = 0; cbl < CH; ++cbl) {
+                    const uint32_t cv = ch * CH + cbl;
+                    if (cv >= nvr) break;
+                    uint32_t pan, pc;
+                    fdivmod32(cv, divq, pan, pc);
+                    E x[V];
+                    unpack<EB>(lds128(sb + pan * p.pstride + (i * q + pc) * 16), x);
+                    char *oc = out + (uint64_t)cbl * V * mEB;
+#pragma unroll
+                    for (uint32_t k = 0; k < V; ++k) *reinterpret_cast<E *>(oc + k * mEB) = x[k];
+                }
+            }
+        });
+}
+
 // ------------------------------------------------- group-split element-path kernel
 // Tiles whose sides are not multiples of 16/elem (e.g. 64 x 9998 or 14803 x 32 floats),
 // 4- and 8-byte elements, over a CTA group as tile_group_db.  A slice is a set of row
@@ -1283,6 +1346,10 @@ static GroupCfg group_search(int64_t A, int64_t B, int eb, uint64_t count, int d
         } else {
             const TmaGeomG t = tma_geom_generic(A, B, eb, K, cs);
             if (t.ok) slice = std::max(slice, t.bytes);
+            if (!cs && (B * eb) % 16 == 0 && env_int("IPT_TILE_GEN_TMAA", 1)) {   // tile_group_tma_elem
+                const TmaGeom te = tma_geom((A + V - 1) / V * V, B, eb, K, false);
+                if (te.ok) slice = std::max(slice, te.bytes);
+            }
         }
         slice = (slice + 127) & ~(size_t)127;
         if ((long)(nb * slice) + kGroupStaticSmem > budget) continue;
@@ -1361,6 +1428,45 @@ bool group_tma_setup(const StageDesc &d, TileParams &p, const GroupCfg &g, CUten
     p.pstride = (uint32_t)t.pstride;
     if (env_int("IPT_DEBUG", 0))
         fprintf(stderr, "[ipt] tile_group_tma q=%u npan=%u rows=%u box=%ux%u\n", t.q, t.npan, t.rows, t.q * V, t.br);
+    return true;
+}
+
+// Tensor map + geometry for tile_group_tma_elem: as group_tma_setup, rows counted in
+// ceil(m / V) blocks (the last one partial), row split only, 16-byte aligned input rows.
+template <int EB>
+bool group_tma_setup_elem(const StageDesc &d, TileParams &p, const GroupCfg &g, CUtensorMap *tm,
+                          size_t *slice, int device) {
+    if (EB != 4 && EB != 8) return false;
+    const int V = 16 / EB;
+    if (g.colsplit || (d.B * EB) % 16 || ((uintptr_t)d.base & 15)) return false;
+    if (d.outer > 1 && d.ostride != d.inner * (int64_t)p.tile_bytes) return false;
+    if (!env_int("IPT_TILE_GEN_TMAA", 1)) return false;
+    const int64_t Ac = (d.A + V - 1) / V * V;                  // rows in whole V-blocks
+    const TmaGeom t = tma_geom(Ac, d.B, EB, g.K, false);
+    if (!t.ok) return false;
+    // the boxes cover whole V-blocks and 128-byte aligned panels: the slice buffers may
+    // grow a little beyond the element layout's, within the opt-in shared memory
+    if (t.bytes > g.slice && (size_t)g.nbuf * t.bytes + 4096 > (size_t)dev_props(device).smem_optin) return false;
+    auto enc = tensor_map_encoder();
+    if (!enc) return false;
+    const uint64_t total_rows = (uint64_t)(d.outer * d.inner) * (uint64_t)d.A;
+    cuuint64_t dims[2] = {(cuuint64_t)d.B, (cuuint64_t)total_rows};
+    cuuint64_t strides[1] = {(cuuint64_t)(d.B * EB)};
+    cuuint32_t box[2] = {t.q * (uint32_t)V, t.br};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(tm, EB == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 2, d.base,
+                     dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) { cudaGetLastError(); return false; }
+    p.q = t.q;
+    p.box_rows = t.br;
+    p.npan = t.npan;
+    p.pstride = (uint32_t)t.pstride;
+    if (t.bytes > *slice) *slice = t.bytes;
+    p.buf_bytes = (uint32_t)*slice;
+    if (env_int("IPT_DEBUG", 0))
+        fprintf(stderr, "[ipt] tile_group_tma_elem q=%u npan=%u rows=%u box=%ux%u slice=%zu\n", t.q, t.npan,
+                t.rows, t.q * V, t.br, *slice);
     return true;
 }
 
@@ -1449,7 +1555,11 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
     }
     auto kern = GENERIC ? tile_group_generic<EB> : tile_group_db<EB>;
     CUtensorMap tmap;
-    const bool tma = GENERIC ? group_tma_setup_generic<EB>(d, p, g, &tmap) : group_tma_setup<EB>(d, p, g, &tmap);
+    // element path with 16-byte aligned input rows: TMA slices + element write-out
+    size_t slice = g.slice;
+    const bool tma_elem = GENERIC && group_tma_setup_elem<EB>(d, p, g, &tmap, &slice, device);
+    const bool tma = tma_elem || (GENERIC ? group_tma_setup_generic<EB>(d, p, g, &tmap)
+                                          : group_tma_setup<EB>(d, p, g, &tmap));
     cudaError_t e = cudaSuccess;
     if (!p.gexit) {
         e = cudaMemsetAsync(ws, 0, (size_t)g.groups * g.nbuf * kGroupCtrStride, st);
@@ -1468,12 +1578,12 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
         }
     };
     set_smem((const void *)kern);
-    auto tkern = GENERIC ? tile_group_generic_tma<EB> : tile_group_tma<EB>;
+    auto tkern = tma_elem ? tile_group_tma_elem<EB> : (GENERIC ? tile_group_generic_tma<EB> : tile_group_tma<EB>);
     if (tma) set_smem((const void *)tkern);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)(g.groups * g.K), 1, 1);
     cfg.blockDim = dim3(512, 1, 1);
-    cfg.dynamicSmemBytes = g.nbuf * g.slice;
+    cfg.dynamicSmemBytes = g.nbuf * slice;
     cfg.stream = st;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeCooperative;

@@ -40,6 +40,12 @@ for env in [{"IPT_SQ_FORCE": "1", "IPT_SQ_TB": "256"}, {"IPT_SQ_FORCE": "1", "IP
             {"IPT_SQ_FORCE": "1", "IPT_SQ_ELEM": "1"}, {"IPT_SQ_FORCE": "1", "IPT_SQ_TMA": "1"}]:
     sq(300, 2, 4, env)
     sq(129, 3, 8, env)
+# element-path group tiles: TMA slices (aligned input rows) and cp.async slices
+for (b, A, B) in [(2, 999, 96), (2, 96, 999)]:
+    a = seeded.values_np(np.arange(b * A * B), 4)
+    t = torch.from_numpy(a.view(np.int32).copy()).cuda()
+    ipt.ipt_010_(t, b, A, B)
+    ok &= np.array_equal(t.cpu().numpy().view(np.uint32), oracle.permute_inplace(a.copy(), b, A, B, 1))
 # segmented cycle following (one grid barrier, no flags)
 os.environ["IPT_CYC_SEG"] = "2"
 for (b, A, B, s) in [(1, 180, 40, 36), (3, 17, 31, 8), (2, 40, 56, 600)]:

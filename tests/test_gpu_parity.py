@@ -1062,3 +1062,30 @@ def test_cycle_seg_counters_across_streams_and_many_launches(monkeypatch):
     torch.cuda.synchronize()
     for k in range(2):
         assert np.array_equal(to_np(ts[k], 4), refs[k].view(np.uint32)), k
+
+
+def test_fuzz_plans_and_kernel_variants(monkeypatch):
+    """Seeded fuzz: random shapes, random valid tilings (m | M, n | N) and random kernel
+    choices (flag / segmented cycles, swizzled / padded square swaps, TMA / cp.async tile
+    slices, self-resetting / memset counters) -- every result bit-exact vs the oracle."""
+    rnd = random.Random(2024)
+
+    def divs(x):
+        return [d for d in range(1, x + 1) if x % d == 0]
+
+    knobs = {"IPT_CYC_SEG": ["0", "1", "2"], "IPT_SQ_SWZ": ["0", "1"],
+             "IPT_TILE_GROUP_TMA": ["0", "1"], "IPT_TILE_GEN_TMAA": ["0", "1"],
+             "IPT_SEG_RESET": ["0", "1"], "IPT_TILE_RESET": ["0", "1"]}
+    for it in range(120):
+        for k, vals in knobs.items():
+            monkeypatch.setenv(k, rnd.choice(vals))
+        eb = rnd.choice([4, 4, 8])
+        M = rnd.choice([rnd.randint(2, 120), rnd.randint(100, 900), rnd.choice([360, 720, 1000, 1024])])
+        N = rnd.choice([M, rnd.randint(2, 120), rnd.randint(100, 900)])
+        m, n = rnd.choice(divs(M)), rnd.choice(divs(N))
+        p = ipt.plan(M, N, eb, 0, m=m, n=n)
+        a = seeded.matrix_np(M, N, eb, seed=seeded.SEED + it)
+        t = to_dev(a, eb)
+        ipt.transpose_(t, M, N, plan_=p)
+        ok = np.array_equal(to_np(t, eb), oracle.transpose_inplace(a.copy(), M, N))
+        assert ok, (it, M, N, m, n, eb, {k: os.environ.get(k) for k in knobs})

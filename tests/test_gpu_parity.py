@@ -1076,7 +1076,7 @@ def test_fuzz_plans_and_kernel_variants(monkeypatch):
     knobs = {"IPT_CYC_SEG": ["0", "1", "2"], "IPT_SQ_SWZ": ["0", "1"],
              "IPT_TILE_GROUP_TMA": ["0", "1"], "IPT_TILE_GEN_TMAA": ["0", "1"],
              "IPT_SEG_RESET": ["0", "1"], "IPT_TILE_RESET": ["0", "1"]}
-    for it in range(120):
+    for it in range(300):
         for k, vals in knobs.items():
             monkeypatch.setenv(k, rnd.choice(vals))
         eb = rnd.choice([4, 4, 8])

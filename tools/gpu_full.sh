@@ -14,7 +14,7 @@ for w in c1 c3 c4 c5; do
   timeout 900 $NCU --nvtx --nvtx-include "timed/" --metrics $M --clock-control none --csv --log-file gpurun_out/launches_$w.csv python bench.py --workload $w --steps 2 --warmup 3 --no-e2e --no-cpu > gpurun_out/launches_bench_$w.log 2>&1
 done
 # one full capture of each kernel kind on sweep matrices (12800x15000 and 9998x12288 plans)
-timeout 900 $NCU --set full --clock-control none --import-source on -k regex:cycle_global -s 1 -c 1 -o gpurun_out/prof_cyc -f python tools/prof_one.py 12800 15000 2 > gpurun_out/prof_cyc.log 2>&1
+IPT_CYC_SEG=0 timeout 900 $NCU --set full --clock-control none --import-source on -k regex:cycle_global -s 1 -c 1 -o gpurun_out/prof_cyc -f python tools/prof_one.py 12800 15000 2 > gpurun_out/prof_cyc.log 2>&1
 timeout 600 $NCU --set full --clock-control none --import-source on -k regex:tile_ -s 2 -c 1 -o gpurun_out/prof_tile -f python tools/prof_one.py 12800 15000 2 > gpurun_out/prof_tile.log 2>&1
 timeout 600 $NCU --set full --clock-control none --import-source on -k regex:tile_ -s 2 -c 1 -o gpurun_out/prof_tile_generic -f python tools/prof_one.py 9998 12288 2 > gpurun_out/prof_tile_generic.log 2>&1
 timeout 600 $NCU --set full --clock-control none --import-source on -k regex:square_swap -s 1 -c 1 -o gpurun_out/prof_sq -f python tools/prof_one.py 16384 16384 2 > gpurun_out/prof_sq.log 2>&1

@@ -195,6 +195,22 @@ ipt_status ipt_transpose_host_pipeline(void *const *h_ptrs, const int64_t *Ms, c
                                        int count, int elem_bytes, void *d_buffer,
                                        size_t d_buffer_bytes, void *stream);
 
+/* ------------------------------------------------------------------- CUDA graphs */
+
+/* Capture the launches of `plan` applied to `count` matrices at d_base (stride_bytes apart;
+ * ignored for count == 1) into an executable CUDA graph; *out receives an opaque handle.
+ * Replaying it (ipt_graph_launch) transposes those matrices in place with one
+ * cudaGraphLaunch -- no per-call planning, validation or kernel-launch overhead.  The graph
+ * is bound to the pointers and the workspace (NULL = an internal buffer owned by the
+ * graph's capture stream).  Lazily built state (segment lists of segmented cycle stages,
+ * self-resetting counters) is used only if it exists already: run the plan once before
+ * capturing to get identical kernels.  Note that an M x N graph replayed twice applies the
+ * M x N transposition twice; pair it with an N x M graph. */
+ipt_status ipt_graph_create(void *d_base, int64_t count, int64_t stride_bytes, const ipt_plan_t *plan,
+                            void *d_workspace, size_t ws_bytes, void **out);
+ipt_status ipt_graph_launch(void *graph, void *stream);
+ipt_status ipt_graph_destroy(void *graph);
+
 /* ------------------------------------------------ elementary transpositions */
 
 /* Device workspace bytes for P(batch, A, B, s) with elem_bytes elements (for s == 1 it

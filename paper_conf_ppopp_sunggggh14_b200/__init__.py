@@ -76,6 +76,9 @@ ABI = [
     ("ipt_transpose_host_async", _int, [_vp, _i64, _i64, _int, _int, _vp, _sz, _vp]),
     ("ipt_transpose_host_pipeline", _int,
      [ctypes.POINTER(_vp), ctypes.POINTER(_i64), ctypes.POINTER(_i64), _int, _int, _vp, _sz, _vp]),
+    ("ipt_graph_create", _int, [_vp, _i64, _i64, ctypes.POINTER(Plan), _vp, _sz, ctypes.POINTER(_vp)]),
+    ("ipt_graph_launch", _int, [_vp, _vp]),
+    ("ipt_graph_destroy", _int, [_vp]),
     ("ipt_stage_workspace_bytes", _sz, [_i64, _i64, _i64, _i64, _int]),
     ("ipt_100", _int, [_vp, _i64, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
     ("ipt_010", _int, [_vp, _i64, _i64, _i64, _int, _vp, _sz, _vp]),
@@ -304,6 +307,32 @@ def transpose_host_pipeline_(hs, shapes, stream=None, elem_bytes: int | None = N
     _check(lib().ipt_transpose_host_pipeline(ptrs, Ms, Ns, n, eb, None, 0, _stream_ptr(stream)),
            "ipt_transpose_host_pipeline")
     return hs
+
+
+class Graph:
+    """A captured CUDA graph of one plan on fixed pointers (ipt_graph_create); launch() replays
+    it on a stream.  Transpose once (uncaptured) before creating it to reuse the same
+    kernels; an M x N graph pairs with an N x M one for repeated use."""
+
+    def __init__(self, t, M: int, N: int, plan_: "Plan | None" = None, count: int = 1,
+                 stride_elems: int | None = None, elem_bytes: int | None = None):
+        eb = _eb(t, elem_bytes)
+        p = plan_ if plan_ is not None else plan(M, N, eb, t.device.index)
+        stride = (stride_elems if stride_elems is not None else M * N) * eb
+        h = ctypes.c_void_p()
+        _check(lib().ipt_graph_create(_dev_ptr(t), count, stride, ctypes.byref(p), None, 0,
+                                      ctypes.byref(h)), "ipt_graph_create")
+        self._h, self._t = h, t
+
+    def launch(self, stream=None):
+        _check(lib().ipt_graph_launch(self._h, _stream_ptr(stream)), "ipt_graph_launch")
+
+    def __del__(self):
+        try:
+            if self._h:
+                lib().ipt_graph_destroy(self._h)
+        except Exception:
+            pass
 
 
 # ----------------------------------------------------------- elementary transpositions

@@ -871,6 +871,74 @@ ipt_status ipt_asta_to_soa(void *d_ptr, int64_t M, int64_t N, int64_t m, int ele
 }
 
 // -------------------------------------------------------------------- diagnostics
+// ---------------------------------------------------------------- CUDA graphs
+// A plan's launches (memsets + 1-3 kernels, or more for batches) captured once into an
+// executable CUDA graph and replayed with one cudaGraphLaunch: no per-call host planning,
+// validation or launch overhead (small matrices are launch-latency sensitive).  Capture
+// runs on an internal stream; state built lazily on a first call (segment lists,
+// self-resetting counters) is only used if it already exists -- transpose once before
+// capturing to get the same kernels as the uncaptured call.
+struct GraphHandle {
+    cudaGraphExec_t exec;
+};
+
+ipt_status ipt_graph_create(void *d_base, int64_t count, int64_t stride_bytes, const ipt_plan_t *plan,
+                            void *d_workspace, size_t ws_bytes, void **out) {
+    if (!out) return IPT_ERR_INVALID_ARG;
+    *out = nullptr;
+    ipt_status s = validate_plan(plan);
+    if (s) return s;
+    if (count < 1) return IPT_ERR_INVALID_ARG;
+    if ((s = check_ptr(d_base, plan->elem_bytes))) return s;
+    const int64_t mat = plan->M * plan->N * plan->elem_bytes;
+    if (count == 1) stride_bytes = mat;
+    if (count > 1 && (stride_bytes < mat || stride_bytes % plan->elem_bytes)) return IPT_ERR_INVALID_ARG;
+    const int device = current_device();
+    if (device < 0) return IPT_ERR_NO_DEVICE;
+    cudaStream_t cs;
+    cudaError_t e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+    if (e != cudaSuccess) return cuda_status(e);
+    void *ws = d_workspace;
+    size_t wsb = ws_bytes;
+    if (!ws) {   // allocate outside the capture (keyed by the capture stream: one per graph)
+        const size_t need = batched_ws(plan, count);
+        if ((s = get_ws(device, (void *)cs, need, &ws))) { cudaStreamDestroy(cs); return s; }
+        wsb = need;
+    }
+    cudaGraph_t g = nullptr;
+    e = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal);
+    if (e == cudaSuccess) {
+        s = run_plan((char *)d_base, count, stride_bytes, plan, ws, wsb, cs, nullptr);
+        cudaError_t e2 = cudaStreamEndCapture(cs, &g);
+        if (!s && e2 != cudaSuccess) e = e2;
+    }
+    GraphHandle *h = nullptr;
+    if (!s && e == cudaSuccess) {
+        h = new GraphHandle{};
+        e = cudaGraphInstantiate(&h->exec, g, 0);
+        if (e != cudaSuccess) { delete h; h = nullptr; }
+    }
+    if (g) cudaGraphDestroy(g);
+    // the capture stream stays alive: the internal workspace and counters are keyed by it
+    if (s) return s;
+    if (e != cudaSuccess) return cuda_status(e);
+    *out = h;
+    return IPT_OK;
+}
+
+ipt_status ipt_graph_launch(void *graph, void *stream) {
+    if (!graph) return IPT_ERR_INVALID_ARG;
+    return cuda_status(cudaGraphLaunch(((GraphHandle *)graph)->exec, (cudaStream_t)stream));
+}
+
+ipt_status ipt_graph_destroy(void *graph) {
+    if (!graph) return IPT_OK;
+    GraphHandle *h = (GraphHandle *)graph;
+    cudaError_t e = cudaGraphExecDestroy(h->exec);
+    delete h;
+    return cuda_status(e);
+}
+
 const char *ipt_status_string(ipt_status s) {
     switch (s) {
         case IPT_OK: return "IPT_OK";

@@ -255,6 +255,9 @@ def main():
                     help="per-stage CUDA events (roofline per-kernel times): every timed step, "
                          "the last two (default: an event record between every stage costs "
                          "2.7 %% on the sweep, 17 %% on 50 MB matrices), or none")
+    ap.add_argument("--graphs", type=int, default=0,
+                    help="1: replay each matrix's plan as a captured CUDA graph (ipt_graph_*) on "
+                         "the steps without per-stage events")
     ap.add_argument("--algo", default="3stage", choices=["3stage", "4stage"],
                     help="4stage = the paper's Gustavson/Karlsson baseline (comparison only)")
     args = ap.parse_args()
@@ -324,11 +327,18 @@ def main():
     ws = torch.empty(max(ws_bytes, 256), dtype=torch.uint8, device=dev)
     orient = [False] * len(mats)   # False: currently M x N; True: currently N x M
 
+    graphs = {}
+
     def one_step(evs=None):
         for i, (t, M, N, cnt, _) in enumerate(mats):
             a, b = (N, M) if orient[i] else (M, N)
             p = plans[(a, b)]
-            if cnt > 1:
+            if args.graphs and evs is None and args.algo == "3stage":
+                key = (i, a, b)          # one captured graph per matrix and orientation
+                if key not in graphs:
+                    graphs[key] = ipt.Graph(t, a, b, p, count=cnt)
+                graphs[key].launch()
+            elif cnt > 1:
                 ipt.transpose_batched_(t, cnt, a, b, plan_=p,
                                        events=evs[i] if evs is not None else None)
             elif args.algo == "4stage":      # the paper's 4-stage baseline

@@ -96,14 +96,18 @@ class NvmlClockSampler:
         self.th = threading.Thread(target=self._run, daemon=True)
         self.th.start()
 
-    def _run(self):
+    def sample(self):
+        """One sample (also called from the main thread while it waits for the GPU)."""
         nv = self.nv
+        try:
+            self.rows.append((nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM),
+                              nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)))
+        except Exception:
+            pass
+
+    def _run(self):
         while not self.stop_ev.is_set():
-            try:
-                self.rows.append((nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM),
-                                  nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)))
-            except Exception:
-                pass
+            self.sample()
             self.stop_ev.wait(0.002)
 
     def stop(self):
@@ -236,7 +240,7 @@ def run_reference(args, world, rank):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="sweep", choices=sorted(WORKLOADS))
@@ -401,7 +405,11 @@ def main():
             step_ev[s][1].record()
     # wait with the GIL released so the clock sampler thread runs during the whole region
     last = t_end if flush is None else step_ev[-1][1]
+    t_poll = 0.0
     while not last.query():
+        if hasattr(clocks, "sample") and time.perf_counter() - t_poll > 0.002:
+            clocks.sample()      # the GPU is still running the timed steps
+            t_poll = time.perf_counter()
         time.sleep(0.0005)
     torch.cuda.synchronize()
     torch.cuda.nvtx.range_pop()

@@ -38,7 +38,11 @@
  *   - Workspace: cycle-following stages need one flag bit per moved unit plus a work
  *     counter ("only one bit per super-element is needed").  Pass a device
  *     buffer of ipt_workspace_bytes() bytes, or NULL to use an internal per-(device,
- *     stream) cache.  libipt zeroes the flags itself before every stage.
+ *     stream) cache (a cached buffer that must grow is retired, never freed, so work or
+ *     graphs already holding it stay valid; under stream capture a NULL workspace is a
+ *     graph-owned allocation instead, see ipt_graph_create).  libipt zeroes the flags
+ *     itself before every stage.  Host-delegated calls (ipt_transpose_host*) refuse
+ *     stream capture (IPT_ERR_INVALID_ARG).
  *   - Thread safety: concurrent calls on distinct buffers with distinct workspaces (or
  *     distinct streams when using the internal cache) are safe.
  *   - M == 1 or N == 1 (and empty batches) are successful no-ops.
@@ -201,11 +205,18 @@ ipt_status ipt_transpose_host_pipeline(void *const *h_ptrs, const int64_t *Ms, c
  * ignored for count == 1) into an executable CUDA graph; *out receives an opaque handle.
  * Replaying it (ipt_graph_launch) transposes those matrices in place with one
  * cudaGraphLaunch -- no per-call planning, validation or kernel-launch overhead.  The graph
- * is bound to the pointers and the workspace (NULL = an internal buffer owned by the
- * graph's capture stream).  Lazily built state (segment lists of segmented cycle stages,
- * self-resetting counters) is used only if it exists already: run the plan once before
- * capturing to get identical kernels.  Note that an M x N graph replayed twice applies the
- * M x N transposition twice; pair it with an N x M graph. */
+ * is bound to the pointers.  Workspace: the caller's d_workspace (>= ipt_workspace_bytes;
+ * then replays must not overlap each other or other calls using it), or NULL = a
+ * graph-owned allocation made and released inside every replay (memory allocation nodes),
+ * so replays on any stream never share flags or counters with other work.  Captured
+ * launches never use the library's per-stream self-resetting counters (they zero their
+ * counters with memset nodes).  Segment lists of segmented cycle stages are used only if a
+ * direct call built them already (else the flag kernel is captured): run the plan once
+ * before capturing to get identical kernels.  ipt_graph_destroy frees everything the
+ * handle owns (the caller synchronises first).  Note that an M x N graph replayed twice
+ * applies the M x N transposition twice; pair it with an N x M graph.
+ * The same rules apply to any libipt call captured by the caller (e.g. torch.cuda.graph):
+ * with a NULL workspace the captured sequence allocates and frees its own flags. */
 ipt_status ipt_graph_create(void *d_base, int64_t count, int64_t stride_bytes, const ipt_plan_t *plan,
                             void *d_workspace, size_t ws_bytes, void **out);
 ipt_status ipt_graph_launch(void *graph, void *stream);

@@ -109,6 +109,8 @@ def lib():
             f = getattr(L, name)
             f.restype = res
             f.argtypes = args
+        L.ipt__stage_kernel.restype = ctypes.c_int
+        L.ipt__stage_kernel.argtypes = [ctypes.POINTER(Plan), _i64, _vp, _int, ctypes.c_char_p, _int]
         L.ipt__fastdiv.restype = ctypes.c_uint64
         L.ipt__fastdiv.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
         L.ipt__fastdiv32.restype = ctypes.c_uint32
@@ -318,11 +320,16 @@ class Graph:
                  stride_elems: int | None = None, elem_bytes: int | None = None):
         eb = _eb(t, elem_bytes)
         p = plan_ if plan_ is not None else plan(M, N, eb, t.device.index)
-        stride = (stride_elems if stride_elems is not None else M * N) * eb
+        if (p.M, p.N, p.elem_bytes) != (M, N, eb):
+            raise IptError(f"plan is for {p.M}x{p.N} ({p.elem_bytes} B), not {M}x{N} ({eb} B)")
+        se = stride_elems if stride_elems is not None else M * N
+        if count < 1 or (count > 1 and se < M * N) or (count - 1) * se + M * N > _nelem(t, eb):
+            raise IptError("tensor too small for the batch (count, stride, M*N)")
+        stride = se * eb
         h = ctypes.c_void_p()
         _check(lib().ipt_graph_create(_dev_ptr(t), count, stride, ctypes.byref(p), None, 0,
                                       ctypes.byref(h)), "ipt_graph_create")
-        self._h, self._t = h, t
+        self._h, self._t, self._plan = h, t, p   # the graph records t's storage: keep it alive
 
     def launch(self, stream=None):
         _check(lib().ipt_graph_launch(self._h, _stream_ptr(stream)), "ipt_graph_launch")
@@ -383,6 +390,19 @@ aos_to_asta_ = _marshal("ipt_aos_to_asta")
 asta_to_aos_ = _marshal("ipt_asta_to_aos")
 soa_to_asta_ = _marshal("ipt_soa_to_asta")
 asta_to_soa_ = _marshal("ipt_asta_to_soa")
+
+
+def stage_kernels(p: Plan, count: int = 1, t=None) -> list:
+    """Names of the kernels the three stages of plan p launch for `count` packed matrices at
+    t's storage (diagnostics: per-kernel attribution of stage times)."""
+    out = []
+    for st in range(3):
+        buf = ctypes.create_string_buffer(64)
+        ptr = ctypes.c_void_p(t.data_ptr()) if t is not None else None
+        if lib().ipt__stage_kernel(ctypes.byref(p), count, ptr, st, buf, 64) != 0:
+            raise IptError("ipt__stage_kernel: invalid plan")
+        out.append(buf.value.decode())
+    return out
 
 
 def kernel_launch_count() -> int:

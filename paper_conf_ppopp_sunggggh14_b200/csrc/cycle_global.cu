@@ -720,6 +720,14 @@ size_t cycle_ws_bytes(const StageDesc &d) {
     return 256 + nwords * 4;
 }
 
+bool cycle_seg_would_launch(const StageDesc &d, int device);   // cycle_seg.cu
+
+const char *cycle_kernel_name(const StageDesc &d, int device) {
+    if (cycle_prefer_seg(d.A * d.B, d.outer * d.inner, d.s * d.eb, device) && cycle_seg_would_launch(d, device))
+        return "cycle_seg";
+    return choose(d).ua ? "cycle_ua" : "cycle_global";
+}
+
 cudaError_t launch_cycle_global(const StageDesc &d, void *ws, cudaStream_t st, int device) {
     // Segmented cycle following (cycle_seg.cu): precomputed equal-length segments, no flags,
     // where the planner's model predicts it faster (IPT_CYC_SEG: 0 never, 2 always).

@@ -28,6 +28,7 @@
 #include "mem_ptx.cuh"
 
 #include <algorithm>
+#include <atomic>
 #include <cstdio>
 #include <cstring>
 #include <map>
@@ -146,6 +147,12 @@ struct SegPlan {
     bool ok = false;
     uint64_t L = 0, nseg = 0;
     void *dev = nullptr;   // ulonglong2[nseg], library-owned, never freed (plan cache)
+    // The list is uploaded asynchronously on the stream of the first call (pinned staging
+    // buffer, event `ready`): a later launch on another stream waits for the event; once it
+    // has been seen complete (`landed`), the staging buffer is freed and no wait is needed.
+    cudaEvent_t ready = nullptr;
+    void *staging = nullptr;
+    std::atomic<bool> landed{false};
 };
 
 // Walk the cycles of k -> (k mod B) * A + k / B on n = A*B units; cut each non-trivial
@@ -256,15 +263,11 @@ std::mutex g_seg_mu;
 std::map<std::tuple<int, uint64_t, uint64_t, uint64_t>, std::shared_ptr<SegPlan>> g_seg_cache;
 
 // Self-resetting barrier counters, one zero-initialised pair per (device, stream); created
-// synchronously on first use (never inside stream capture), never freed.
+// on first use, never freed.  Never used by captured launches: a graph may be replayed on
+// another stream concurrently with direct calls on this one (the workspace + memset path
+// is captured instead).
 std::mutex g_ctr_mu;
 std::map<std::pair<int, cudaStream_t>, unsigned int *> g_ctr;
-
-unsigned int *seg_counters_cached(int device, cudaStream_t st) {
-    std::lock_guard<std::mutex> lk(g_ctr_mu);
-    auto it = g_ctr.find(std::make_pair(device, st));
-    return it == g_ctr.end() ? nullptr : it->second;
-}
 
 unsigned int *seg_counters(int device, cudaStream_t st) {
     std::lock_guard<std::mutex> lk(g_ctr_mu);
@@ -287,7 +290,7 @@ bool seg_plan_cached(int device, uint64_t A, uint64_t B, uint64_t max_seg) {
     return g_seg_cache.count(std::make_tuple(device, A, B, max_seg)) != 0;
 }
 
-std::shared_ptr<SegPlan> seg_plan(int device, uint64_t A, uint64_t B, uint64_t max_seg) {
+std::shared_ptr<SegPlan> seg_plan(int device, uint64_t A, uint64_t B, uint64_t max_seg, cudaStream_t st) {
     const auto key = std::make_tuple(device, A, B, max_seg);
     {
         std::lock_guard<std::mutex> lk(g_seg_mu);
@@ -301,21 +304,46 @@ std::shared_ptr<SegPlan> seg_plan(int device, uint64_t A, uint64_t B, uint64_t m
         sp->L = L;
         sp->nseg = segs.size();
         sp->ok = true;
+        sp->landed = segs.empty();
         if (!segs.empty()) {
-            // cudaMemcpy from pageable memory may return before the DMA lands, and a
-            // non-blocking stream is not ordered after it: wait for it (once per shape)
-            if (cudaMalloc(&sp->dev, segs.size() * sizeof(ulonglong2)) != cudaSuccess ||
-                cudaMemcpy(sp->dev, segs.data(), segs.size() * sizeof(ulonglong2),
-                           cudaMemcpyHostToDevice) != cudaSuccess ||
-                cudaDeviceSynchronize() != cudaSuccess) {
+            // asynchronous upload on the caller's stream: no host stall on unrelated device
+            // work (the first call of a shape may come from an asynchronous API)
+            const size_t bytes = segs.size() * sizeof(ulonglong2);
+            if (cudaMalloc(&sp->dev, bytes) != cudaSuccess || cudaMallocHost(&sp->staging, bytes) != cudaSuccess ||
+                cudaEventCreateWithFlags(&sp->ready, cudaEventDisableTiming) != cudaSuccess) {
                 cudaGetLastError();
                 sp->ok = false;
+            } else {
+                std::memcpy(sp->staging, segs.data(), bytes);
+                if (cudaMemcpyAsync(sp->dev, sp->staging, bytes, cudaMemcpyHostToDevice, st) != cudaSuccess ||
+                    cudaEventRecord(sp->ready, st) != cudaSuccess) {
+                    cudaGetLastError();
+                    sp->ok = false;
+                }
             }
         }
     }
     std::lock_guard<std::mutex> lk(g_seg_mu);
     g_seg_cache[key] = sp;
     return sp;
+}
+
+// Order a launch on `st` after the plan's upload.  Returns false when that cannot be done
+// under stream capture (upload not yet seen complete): the caller uses the flag kernel.
+bool seg_plan_ready(SegPlan &sp, cudaStream_t st, bool capturing) {
+    if (sp.landed) return true;
+    std::lock_guard<std::mutex> lk(g_seg_mu);
+    if (sp.landed) return true;
+    if (capturing) return false;
+    const cudaError_t q = cudaEventQuery(sp.ready);
+    if (q == cudaSuccess) {
+        cudaFreeHost(sp.staging);
+        sp.staging = nullptr;
+        sp.landed = true;
+        return true;
+    }
+    cudaGetLastError();   // cudaErrorNotReady
+    return cudaStreamWaitEvent(st, sp.ready, 0) == cudaSuccess;
 }
 
 }  // namespace
@@ -362,9 +390,10 @@ cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int 
     if (cudaStreamIsCapturing(st, &cap) != cudaSuccess) { cudaGetLastError(); cap = cudaStreamCaptureStatusActive; }
     if (cap != cudaStreamCaptureStatusNone && !seg_plan_cached(device, (uint64_t)d.A, (uint64_t)d.B, per_item))
         return cudaErrorNotSupported;
-    auto sp = seg_plan(device, (uint64_t)d.A, (uint64_t)d.B, per_item);
+    auto sp = seg_plan(device, (uint64_t)d.A, (uint64_t)d.B, per_item, st);
     if (!sp->ok) return cudaErrorNotSupported;
     if (sp->nseg == 0) return cudaSuccess;   // identity permutation
+    if (!seg_plan_ready(*sp, st, cap != cudaStreamCaptureStatusNone)) return cudaErrorNotSupported;
     SegParams p{};
     p.base = d.base;
     p.ostride = (uint64_t)d.ostride;
@@ -388,7 +417,7 @@ cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int 
     // with a memset when the pair cannot be created (e.g. first use inside stream capture)
     unsigned int *ctr = nullptr;
     if (env_int("IPT_SEG_RESET", 1))
-        ctr = cap == cudaStreamCaptureStatusNone ? seg_counters(device, st) : seg_counters_cached(device, st);
+        ctr = cap == cudaStreamCaptureStatusNone ? seg_counters(device, st) : nullptr;   // captured: workspace
     cudaError_t e = cudaSuccess;
     if (ctr) {
         p.bar = ctr;
@@ -414,6 +443,19 @@ cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int 
     }
     note_launch();
     return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+// Would launch_cycle_seg run this stage (diagnostics)?  Without a cached segment plan the
+// cycles are not walked here: a stage with more cycles than walkers (rare) is reported as
+// segmented although the launcher then falls back to the flag kernel.
+bool cycle_seg_would_launch(const StageDesc &d, int device) {
+    if (!cycle_seg_applicable(d)) return false;
+    const SegCfg c = seg_cfg((uint64_t)(d.s * d.eb));
+    const int per_sm = seg_blocks_per_sm(seg_kernel(c.G, c.R));
+    if (per_sm < 1) return false;
+    const uint64_t items = (uint64_t)(d.outer * d.inner);
+    const uint64_t walkers = (uint64_t)dev_props(device).sms * per_sm * 256 / c.G;
+    return walkers / (items * c.nch) >= 1;
 }
 
 // Planner estimate of the segment length L (units per walker) without walking cycles.

@@ -141,8 +141,20 @@ WsCache &ws_cache() {
 }
 
 // Internal buffers are cached per (device, stream, purpose): `purpose` 0 = flag workspace,
-// 1 = host-path staging buffer, 2 = host pipeline buffers.  Growing a buffer synchronises `stream` first (work
-// already enqueued on it may still use the old buffer).
+// 1 = host-path staging buffer, 2 = host pipeline buffers.  A flag workspace that must grow
+// is RETIRED, not freed: work already enqueued on the stream -- or a CUDA graph captured
+// from it by the caller -- may still hold the old pointer, so it stays valid until process
+// exit (flag workspaces are small: one bit per unit).  Staging buffers (whole
+// matrices) are freed after synchronising the stream; the host paths refuse stream capture.
+bool stream_capturing(cudaStream_t st) {
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(st, &cap) != cudaSuccess) {
+        cudaGetLastError();
+        return true;   // unknown: treat as capturing (no synchronising calls)
+    }
+    return cap != cudaStreamCaptureStatusNone;
+}
+
 ipt_status get_ws(int device, void *stream, size_t need, void **out, int purpose = 0) {
     if (need == 0) { *out = nullptr; return IPT_OK; }
     WsCache &c = ws_cache();
@@ -154,8 +166,11 @@ ipt_status get_ws(int device, void *stream, size_t need, void **out, int purpose
         return IPT_OK;
     }
     if (it != c.bufs.end()) {
-        cudaStreamSynchronize((cudaStream_t)stream);
-        cudaFree(it->second.first);
+        if (purpose != 0) {
+            if (stream_capturing((cudaStream_t)stream)) return IPT_ERR_INVALID_ARG;
+            cudaStreamSynchronize((cudaStream_t)stream);
+            cudaFree(it->second.first);
+        }   // purpose 0: retired, never freed (see above)
         c.bufs.erase(it);
     }
     size_t sz = need < (1u << 20) ? (1u << 20) : need + need / 4;
@@ -167,6 +182,38 @@ ipt_status get_ws(int device, void *stream, size_t need, void **out, int purpose
     c.bufs[key] = std::make_pair(p, sz);
     *out = p;
     return IPT_OK;
+}
+
+// Flag workspace of one call: the caller's (checked), else a graph-owned allocation under
+// stream capture (released by release_ws at the end of the captured sequence), else the
+// per-stream cache.
+struct CallWs {
+    void *ptr = nullptr;
+    bool graph_owned = false;
+};
+
+ipt_status acquire_ws(int device, cudaStream_t st, size_t need, void *user, size_t user_bytes, CallWs *w) {
+    w->graph_owned = false;
+    if (user) {
+        if (user_bytes < need) return IPT_ERR_NO_MEMORY;
+        w->ptr = user;
+        return IPT_OK;
+    }
+    if (need && stream_capturing(st)) {
+        if (cudaMallocAsync(&w->ptr, need, st) != cudaSuccess) {
+            cudaGetLastError();
+            return IPT_ERR_NO_MEMORY;
+        }
+        w->graph_owned = true;
+        return IPT_OK;
+    }
+    return get_ws(device, (void *)st, need, &w->ptr);
+}
+
+cudaError_t release_ws(const CallWs &w, cudaStream_t st, cudaError_t e) {
+    if (!w.graph_owned) return e;
+    const cudaError_t f = cudaFreeAsync(w.ptr, st);
+    return e != cudaSuccess ? e : f;
 }
 
 thread_local cudaError_t g_last_cuda = cudaSuccess;
@@ -203,12 +250,17 @@ ipt_status validate_plan(const ipt_plan_t *p) {
     if (p->m < 1 || p->n < 1 || p->M % p->m || p->N % p->n || p->Mp != p->M / p->m ||
         p->Np != p->N / p->n)
         return IPT_ERR_INVALID_ARG;
-    for (int i = 0; i < 3; ++i)
-        if (p->variant[i] < IPT_VAR_IDENTITY || p->variant[i] > IPT_VAR_SQUARE_SWAP)
-            return IPT_ERR_INVALID_ARG;
-    if ((p->variant[0] == IPT_VAR_SQUARE_SWAP || p->variant[2] == IPT_VAR_SQUARE_SWAP) ||
-        (p->variant[1] == IPT_VAR_SQUARE_SWAP && p->m != p->n))
-        return IPT_ERR_INVALID_ARG;   // only stage 2 with square tiles is a swap
+    // Stage 1 P(1, M, N', n) and stage 3 P(N', M', n, m) move super-elements by cycle
+    // following; stage 2 P(N'M', m, n, 1) is tile-local (on chip, square swap, or cycle
+    // following when the tile does not fit).  A stage may be the identity only when one of
+    // its swapped dimensions is 1 -- a plan edited otherwise is rejected.
+    const int *v = p->variant;
+    const bool id1 = p->M == 1 || p->Np == 1, id2 = p->m == 1 || p->n == 1, id3 = p->Mp == 1 || p->n == 1;
+    if (!(v[0] == IPT_VAR_CYCLE_GLOBAL || (v[0] == IPT_VAR_IDENTITY && id1))) return IPT_ERR_INVALID_ARG;
+    if (!(v[2] == IPT_VAR_CYCLE_GLOBAL || (v[2] == IPT_VAR_IDENTITY && id3))) return IPT_ERR_INVALID_ARG;
+    if (!(v[1] == IPT_VAR_CYCLE_GLOBAL || v[1] == IPT_VAR_TILE_ONCHIP ||
+          (v[1] == IPT_VAR_SQUARE_SWAP && p->m == p->n) || (v[1] == IPT_VAR_IDENTITY && id2)))
+        return IPT_ERR_INVALID_ARG;
     return IPT_OK;
 }
 
@@ -228,28 +280,28 @@ ipt_status run_plan(char *base, int64_t count, int64_t stride, const ipt_plan_t 
     const int device = current_device();
     if (device < 0) return IPT_ERR_NO_DEVICE;
     const size_t need = batched_ws(p, count);
-    if (ws == nullptr) {
-        ipt_status s = get_ws(device, (void *)st, need, &ws);
-        if (s) return s;
-    } else if (ws_bytes < need) {
-        return IPT_ERR_NO_MEMORY;
-    }
+    // Under stream capture (e.g. torch.cuda.graph) without a caller workspace, the flags
+    // live in a graph-owned allocation (cudaMallocAsync / cudaFreeAsync nodes): every
+    // replay gets its own workspace, so replays on other streams never share flags or
+    // counters with direct calls on the capture stream.
+    CallWs w;
+    if (ipt_status s = acquire_ws(device, st, need, ws, ws_bytes, &w)) return s;
+    ws = w.ptr;
     StageDesc sd[3];
     plan_stages(p, base, count, stride, sd);
     rec(events, 0, st);
-    for (int i = 0; i < 3; ++i) {
-        cudaError_t e = cudaSuccess;
+    cudaError_t e = cudaSuccess;
+    for (int i = 0; i < 3 && e == cudaSuccess; ++i) {
         switch (p->variant[i]) {
             case IPT_VAR_IDENTITY: break;
             case IPT_VAR_TILE_ONCHIP: e = launch_tile_onchip(sd[i], ws, st, device); break;
             case IPT_VAR_SQUARE_SWAP: e = launch_square_swap(sd[i], st, device); break;
-            case IPT_VAR_CYCLE_ONCHIP:   // not built yet: global-flag cycle following
             case IPT_VAR_CYCLE_GLOBAL: e = launch_cycle_global(sd[i], ws, st, device); break;
+            default: e = cudaErrorInvalidValue; break;
         }
-        if (e != cudaSuccess) return cuda_status(e);
-        rec(events, i + 1, st);
+        if (e == cudaSuccess) rec(events, i + 1, st);
     }
-    return IPT_OK;
+    return cuda_status(release_ws(w, st, e));
 }
 
 ipt_status check_ptr(const void *p, int eb) {
@@ -388,13 +440,10 @@ static ipt_status run_cycle(void *d, int64_t batch, int64_t A, int64_t B, int64_
     const int device = current_device();
     if (device < 0) return IPT_ERR_NO_DEVICE;
     StageDesc sd = stage_desc(d, batch, A, B, s, eb);
-    const size_t need = cycle_ws_bytes(sd);
-    if (!ws) {
-        if ((st = get_ws(device, stream, need, &ws))) return st;
-    } else if (ws_bytes < need) {
-        return IPT_ERR_NO_MEMORY;
-    }
-    return cuda_status(launch_cycle_global(sd, ws, (cudaStream_t)stream, device));
+    CallWs w;
+    if ((st = acquire_ws(device, (cudaStream_t)stream, cycle_ws_bytes(sd), ws, ws_bytes, &w))) return st;
+    return cuda_status(release_ws(w, (cudaStream_t)stream,
+                                  launch_cycle_global(sd, w.ptr, (cudaStream_t)stream, device)));
 }
 
 ipt_status ipt_100(void *d_ptr, int64_t batch, int64_t A, int64_t B, int64_t s, int elem_bytes,
@@ -415,13 +464,10 @@ ipt_status ipt_010(void *d_ptr, int64_t batch, int64_t A, int64_t B, int elem_by
     }
     if (tile_onchip_fits(A, B, elem_bytes, device)) {
         StageDesc sd = stage_desc(d_ptr, batch, A, B, 1, elem_bytes);
-        void *ws = d_workspace;
-        if (!ws) {
-            if ((st = get_ws(device, stream, kTileWsBytes, &ws))) return st;
-        } else if (ws_bytes < kTileWsBytes) {
-            return IPT_ERR_NO_MEMORY;
-        }
-        return cuda_status(launch_tile_onchip(sd, ws, (cudaStream_t)stream, device));
+        CallWs w;
+        if ((st = acquire_ws(device, (cudaStream_t)stream, kTileWsBytes, d_workspace, ws_bytes, &w))) return st;
+        return cuda_status(release_ws(w, (cudaStream_t)stream,
+                                      launch_tile_onchip(sd, w.ptr, (cudaStream_t)stream, device)));
     }
     return run_cycle(d_ptr, batch, A, B, 1, elem_bytes, d_workspace, ws_bytes, stream);
 }
@@ -585,20 +631,17 @@ ipt_status ipt_transpose_4stage(void *d_ptr, int64_t M, int64_t N, int64_t m, in
         }
         need = std::max(need, cycle_ws_bytes(sd[i]));
     }
-    void *ws = d_workspace;
-    if (!ws) {
-        if ((s = get_ws(device, stream, need, &ws))) return s;
-    } else if (ws_bytes < need) {
-        return IPT_ERR_NO_MEMORY;
-    }
-    for (int i = 0; i < 4; ++i) {
+    CallWs w;
+    if ((s = acquire_ws(device, (cudaStream_t)stream, need, d_workspace, ws_bytes, &w))) return s;
+    void *ws = w.ptr;
+    cudaError_t e = cudaSuccess;
+    for (int i = 0; i < 4 && e == cudaSuccess; ++i) {
         if (sd[i].A == 1 || sd[i].B == 1) continue;
-        cudaError_t e = (i == 1 && sq2)     ? launch_square_swap(sd[i], (cudaStream_t)stream, device)
-                        : (i == 1 && tile2) ? launch_tile_onchip(sd[i], ws, (cudaStream_t)stream, device)
-                                            : launch_cycle_global(sd[i], ws, (cudaStream_t)stream, device);
-        if (e != cudaSuccess) return cuda_status(e);
+        e = (i == 1 && sq2)     ? launch_square_swap(sd[i], (cudaStream_t)stream, device)
+            : (i == 1 && tile2) ? launch_tile_onchip(sd[i], ws, (cudaStream_t)stream, device)
+                                : launch_cycle_global(sd[i], ws, (cudaStream_t)stream, device);
     }
-    return IPT_OK;
+    return cuda_status(release_ws(w, (cudaStream_t)stream, e));
 }
 
 // ------------------------------------------------- host-delegated transposition (Sec. 6)
@@ -639,6 +682,7 @@ static ipt_status transpose_host_impl(void *h_ptr, int64_t M, int64_t N, int ele
     if (M == 1 || N == 1) return IPT_OK;
     const int device = current_device();
     if (device < 0) return IPT_ERR_NO_DEVICE;
+    if (stream_capturing((cudaStream_t)stream)) return IPT_ERR_INVALID_ARG;
     ipt_plan_t p;
     if ((s = ipt_plan(M, N, elem_bytes, device, &p))) return s;
     const int64_t Np = p.Np;
@@ -754,6 +798,7 @@ ipt_status ipt_transpose_host_pipeline(void *const *h_ptrs, const int64_t *Ms, c
     }
     const int device = current_device();
     if (device < 0) return IPT_ERR_NO_DEVICE;
+    if (stream_capturing((cudaStream_t)stream)) return IPT_ERR_INVALID_ARG;
     std::vector<ipt_plan_t> plans(count);
     size_t ws = 0;
     for (int i = 0; i < count; ++i) {
@@ -895,20 +940,16 @@ ipt_status ipt_graph_create(void *d_base, int64_t count, int64_t stride_bytes, c
     if (count > 1 && (stride_bytes < mat || stride_bytes % plan->elem_bytes)) return IPT_ERR_INVALID_ARG;
     const int device = current_device();
     if (device < 0) return IPT_ERR_NO_DEVICE;
+    if (d_workspace && ws_bytes < batched_ws(plan, count)) return IPT_ERR_NO_MEMORY;
     cudaStream_t cs;
     cudaError_t e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
     if (e != cudaSuccess) return cuda_status(e);
-    void *ws = d_workspace;
-    size_t wsb = ws_bytes;
-    if (!ws) {   // allocate outside the capture (keyed by the capture stream: one per graph)
-        const size_t need = batched_ws(plan, count);
-        if ((s = get_ws(device, (void *)cs, need, &ws))) { cudaStreamDestroy(cs); return s; }
-        wsb = need;
-    }
+    // without a caller workspace, run_plan gives the graph its own workspace (allocation
+    // nodes); library-owned per-stream counters are never used under capture
     cudaGraph_t g = nullptr;
     e = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal);
     if (e == cudaSuccess) {
-        s = run_plan((char *)d_base, count, stride_bytes, plan, ws, wsb, cs, nullptr);
+        s = run_plan((char *)d_base, count, stride_bytes, plan, d_workspace, ws_bytes, cs, nullptr);
         cudaError_t e2 = cudaStreamEndCapture(cs, &g);
         if (!s && e2 != cudaSuccess) e = e2;
     }
@@ -919,7 +960,7 @@ ipt_status ipt_graph_create(void *d_base, int64_t count, int64_t stride_bytes, c
         if (e != cudaSuccess) { delete h; h = nullptr; }
     }
     if (g) cudaGraphDestroy(g);
-    // the capture stream stays alive: the internal workspace and counters are keyed by it
+    cudaStreamDestroy(cs);   // nothing was launched on it: captured work lives in the graph
     if (s) return s;
     if (e != cudaSuccess) return cuda_status(e);
     *out = h;
@@ -957,6 +998,28 @@ uint64_t ipt_kernel_launch_count(void) { return g_launches.load(); }
 const char *ipt_last_cuda_error(void) { return cudaGetErrorString(g_last_cuda); }
 
 const char *ipt_version(void) { return "libipt 0.1 (sm_100a)"; }
+
+// Diagnostic hook (not in the ABI): the kernel stage `stage` (0..2) of `plan` applied to
+// `count` packed matrices at `d_base` launches ("identity", "cycle_global", "cycle_ua",
+// "cycle_seg", "tile_group_tma", "square_swap_vec", ...), copied into buf.  Used by the
+// bench to attribute per-stage event times to kernels (the roofline's dominant kernel).
+int ipt__stage_kernel(const ipt_plan_t *plan, int64_t count, const void *d_base, int stage, char *buf,
+                      int len) {
+    if (validate_plan(plan) || stage < 0 || stage > 2 || !buf || len < 1 || count < 1) return -1;
+    const int device = current_device();
+    StageDesc sd[3];
+    plan_stages(plan, (char *)d_base, count, plan->M * plan->N * plan->elem_bytes, sd);
+    const char *name = "identity";
+    switch (plan->variant[stage]) {
+        case IPT_VAR_TILE_ONCHIP: name = tile_kernel_name(sd[stage], device); break;
+        case IPT_VAR_SQUARE_SWAP: name = square_kernel_name(sd[stage]); break;
+        case IPT_VAR_CYCLE_ONCHIP:
+        case IPT_VAR_CYCLE_GLOBAL: name = cycle_kernel_name(sd[stage], device); break;
+        default: break;
+    }
+    snprintf(buf, (size_t)len, "%s", name);
+    return 0;
+}
 
 // Internal self-test hook (not in the ABI): the multiply-high division used by every
 // kernel's index map, evaluated on the host.

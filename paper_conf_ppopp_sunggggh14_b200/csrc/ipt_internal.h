@@ -107,7 +107,11 @@ bool tile_group_split(int64_t A, int64_t B, int eb, int device);
 bool tile_group_generic_split(int64_t A, int64_t B, int eb, int device);
 // Group split of `count` tiles: CTAs per tile (0 = does not fit) and groups in flight.
 int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups,
-                 bool *tma = nullptr);
+                 bool *tma = nullptr, int *nbuf = nullptr);
+// Kernel names the launchers will run for a stage (diagnostics, ipt__stage_kernel).
+const char *tile_kernel_name(const StageDesc &d, int device);
+const char *cycle_kernel_name(const StageDesc &d, int device);
+const char *square_kernel_name(const StageDesc &d);
 // Workspace of a tile stage: the group split's arrival counters (one per group and slice
 // buffer, kGroupCtrStride bytes apart, at most 256).  `ws` may be NULL for the other paths.
 constexpr uint32_t kGroupCtrStride = 32;

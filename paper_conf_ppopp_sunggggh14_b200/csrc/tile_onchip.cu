@@ -1314,14 +1314,27 @@ static int group_nbuf() {
 
 // Best K for one split direction; `generic`: element-path slices of row pieces with one
 // padding vector (the aligner may read one vector past the last row).
+static GroupCfg group_search_nb(int64_t A, int64_t B, int eb, uint64_t count, int device, bool cs,
+                                bool generic, int nb);
+
+// Double-buffered slices when they fit; otherwise ONE buffer per CTA (no overlap of a
+// tile's write-out with the next tile's fetch, but twice the on-chip capacity: tiles of up
+// to ~33 MB over all 148 SMs -- e.g. a whole 1009 x 7001 float32 matrix in one pass).
 static GroupCfg group_search(int64_t A, int64_t B, int eb, uint64_t count, int device, bool cs,
                              bool generic) {
+    GroupCfg g = group_search_nb(A, B, eb, count, device, cs, generic, group_nbuf());
+    if (!g.K && env_int("IPT_TILE_GROUP_SINGLE", 1))
+        g = group_search_nb(A, B, eb, count, device, cs, generic, 1);
+    return g;
+}
+
+static GroupCfg group_search_nb(int64_t A, int64_t B, int eb, uint64_t count, int device, bool cs,
+                                bool generic, int nb) {
     GroupCfg g;
     const DevProps dp = dev_props(device);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
     const int V = 16 / eb;
     const int kfix = (int)env_int("IPT_TILE_GROUP_K", 0);
-    const int nb = group_nbuf();
     const uint64_t cnt = std::max<uint64_t>(count, 1);
     g.nbuf = nb;
     g.colsplit = cs;
@@ -1505,7 +1518,9 @@ bool group_tma_setup_generic(const StageDesc &d, TileParams &p, const GroupCfg &
 
 // Library-owned group counters per (device, stream): arrivals (kTileWsBytes) then per-group
 // exit counters (kTileWsBytes), zeroed once ON that stream, re-zeroed by each launch's last
-// CTA of every group.  Not created during stream capture (create == false).
+// CTA of every group.  Never used by captured launches (create == false -> the call's
+// workspace with a memset node): a graph may be replayed on another stream concurrently
+// with direct calls on the capture stream.
 static uint32_t *group_counters(int device, cudaStream_t st, bool create) {
     static std::mutex mu;
     static std::map<std::pair<int, cudaStream_t>, uint32_t *> cache;
@@ -1548,7 +1563,7 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
     if (env_int("IPT_TILE_RESET", 1)) {
         cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
         if (cudaStreamIsCapturing(st, &cap) != cudaSuccess) { cudaGetLastError(); cap = cudaStreamCaptureStatusActive; }
-        if (uint32_t *c = group_counters(device, st, cap == cudaStreamCaptureStatusNone)) {
+        if (uint32_t *c = cap == cudaStreamCaptureStatusNone ? group_counters(device, st, true) : nullptr) {
             p.gbar = c;
             p.gexit = c + kTileWsBytes / 4;
         }
@@ -1696,11 +1711,13 @@ bool tile_group_generic_split(int64_t A, int64_t B, int eb, int device) {
     return group_cfg_generic(A, B, eb, (uint64_t)dev_props(device).sms, device).K != 0;
 }
 
-int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups, bool *tma) {
+int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups, bool *tma,
+                 int *nbuf) {
     const bool fast = vec_ok(A, B, eb);
     const GroupCfg g = fast ? group_cfg(A, B, eb, count, device)
                             : group_cfg_generic(A, B, eb, count, device);
     if (groups) *groups = g.groups;
+    if (nbuf) *nbuf = g.nbuf;
     if (tma) *tma = fast && g.K && tma_geom(A, B, eb, g.K, g.colsplit).ok;
     return g.K;
 }
@@ -1717,11 +1734,47 @@ int tile_onchip_path(int64_t A, int64_t B, int eb, int device) {
     return 0;
 }
 
+// Name of the kernel launch_tile_onchip runs for this stage (diagnostics: the bench's
+// per-kernel roofline and the ncu launch lists use the same names).  Mirrors the launcher's
+// decisions; the TMA choices are made on geometry (a tensor-map encode failure at launch
+// falls back to the cp.async kernel of the same family).
+const char *tile_kernel_name(const StageDesc &d, int device) {
+    const DevProps dp = dev_props(device);
+    const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
+    if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) <= budget) {
+        const size_t smem = fast_smem(d.A, d.B, d.eb);
+        if (smem > 113 * 1024 && env_int("IPT_TILE_STREAM", 1) && tile_mode() != MODE_TMA)
+            return "tile_onchip_stream";
+        return tile_mode() == MODE_TMA ? "tile_onchip_tma" : "tile_onchip_ldg";
+    }
+    const uint64_t count = (uint64_t)(d.outer * d.inner);
+    const bool packed = d.outer <= 1 || d.ostride == d.inner * d.A * d.B * d.eb;
+    if (fast_ok(d) && tile_group_split(d.A, d.B, d.eb, device)) {
+        const GroupCfg g = group_cfg(d.A, d.B, d.eb, count, device);
+        const TmaGeom t = tma_geom(d.A, d.B, d.eb, g.K, g.colsplit);
+        return (packed && t.ok && t.bytes <= g.slice) ? "tile_group_tma" : "tile_group_db";
+    }
+    if (!fast_ok(d) && tile_group_generic_split(d.A, d.B, d.eb, device)) {
+        const GroupCfg g = group_cfg_generic(d.A, d.B, d.eb, count, device);
+        const int V = 16 / d.eb;
+        if (!g.colsplit && (d.B * d.eb) % 16 == 0 && ((uintptr_t)d.base & 15) == 0 && packed &&
+            env_int("IPT_TILE_GEN_TMAA", 1) && tma_geom((d.A + V - 1) / V * V, d.B, d.eb, g.K, false).ok)
+            return "tile_group_tma_elem";
+        const TmaGeomG t = tma_geom_generic(d.A, d.B, d.eb, g.K, g.colsplit);
+        return (packed && t.ok && t.bytes <= g.slice) ? "tile_group_generic_tma" : "tile_group_generic";
+    }
+    if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) > budget && tile_cluster_k(d.A, d.B, d.eb, device))
+        return "tile_onchip_cluster";
+    if ((long)generic_smem(d.A, d.B, d.eb) > budget) return "tile_generic_cluster";
+    return "tile_onchip_generic";
+}
+
 bool tile_onchip_fits(int64_t A, int64_t B, int eb, int device) {
     return tile_onchip_path(A, B, eb, device) != 0;
 }
 
 cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, int device) {
+    if (d.s != 1) return cudaErrorInvalidValue;   // tile-local transposition of elements only
     DevProps dp = dev_props(device);
     TileParams p{};
     p.base = d.base;

@@ -178,7 +178,8 @@ def test_workspace_batch_scales():
 
 def test_group_split_extends_on_chip_tiles():
     """Tiles beyond 16 x 227 KB clusters run on chip over co-resident CTA groups (up to
-    ~148 x 113 KB, double-buffered); larger tiles fall back to cycle following.  A tile
+    ~148 x 113 KB double-buffered, ~148 x 227 KB single-buffered); larger tiles fall back to
+    cycle following.  A tile
     stage reserves 8 KB of workspace for the group counters (nominal B200, no GPU)."""
     V = ipt.VARIANTS
     for (M, N, m, n) in [(4096, 8192, 1024, 1024 + 1024),  # 8 MB 16-byte-path tiles
@@ -188,7 +189,10 @@ def test_group_split_extends_on_chip_tiles():
         p = ipt.plan(M, N, 4, m=m, n=n)
         assert V[p.variant[1]] == "tile_onchip", (M, N, m, n)
         assert p.workspace_bytes >= 8192
-    p = ipt.plan(4096, 8192, 4, m=4096, n=2048)         # 32 MB: beyond aggregate smem
+    # up to ~148 x 227 KB with ONE slice buffer per CTA (single-buffered groups)
+    p = ipt.plan(4096, 8192, 4, m=4096, n=2048)         # 32 MB: single-buffered group
+    assert V[p.variant[1]] == "tile_onchip"
+    p = ipt.plan(8192, 8192, 4, m=8192, n=2048)         # 64 MB: beyond aggregate smem
     assert V[p.variant[1]] == "cycle_global"
     assert ipt.lib().ipt_stage_workspace_bytes(3, 120, 7200, 1, 4) >= 8192
     assert ipt.lib().ipt_stage_workspace_bytes(1, 4, 4, 5, 4) < 8192   # cycle stage: flags only

@@ -721,10 +721,11 @@ size_t cycle_ws_bytes(const StageDesc &d) {
 }
 
 bool cycle_seg_would_launch(const StageDesc &d, int device);   // cycle_seg.cu
+const char *cycle_seg_name(const StageDesc &d);
 
 const char *cycle_kernel_name(const StageDesc &d, int device) {
     if (cycle_prefer_seg(d.A * d.B, d.outer * d.inner, d.s * d.eb, device) && cycle_seg_would_launch(d, device))
-        return "cycle_seg";
+        return cycle_seg_name(d);
     return choose(d).ua ? "cycle_ua" : "cycle_global";
 }
 

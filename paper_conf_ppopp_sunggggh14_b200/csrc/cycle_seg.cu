@@ -140,6 +140,173 @@ __global__ void __launch_bounds__(256, 4) cycle_seg_kernel(const SegParams p) {
     }
 }
 
+// ------------------------------------------------- unaligned units (S % 16 != 0, S % 4 == 0)
+// Same schedule for units whose start addresses have different 16-byte phases (e.g.
+// m = 127 floats: 508-byte units).  A walker is a group of G lanes (G | 32; several walkers
+// per warp for small units) holding one chunk of a unit as the 16-byte vectors COVERING it
+// at its source position (vector v = r*G + gl), plus the chunk's word phase o (0..3) there.
+// Storing into a target of phase p shifts the carried words by d = p - o words across the
+// vector frame (one funnel step between neighbouring vectors: a shuffle inside the group,
+// the group's edge lanes taking the neighbouring register); interior vectors are written
+// with 16-byte stores, the two edge vectors word by word (their other words belong to the
+// neighbouring units, moved by their own walkers).  The backup loaded from the target (its
+// covering vectors, phase p) becomes the carried chunk.  Walkers of a warp may diverge
+// (different segment lengths / shifts): every shuffle uses the walker's own lane mask.
+// Vector v + dir (dir = +-1) of the group's frame, for v = r*G + gl.
+template <int G, int R>
+__device__ __forceinline__ uint4 group_vec_nb(const uint4 (&a)[R], int r, uint32_t gl, int dir, unsigned gmask) {
+    const int src = ((int)gl + dir + G) % G;
+    const bool wrap = (int)gl + dir < 0 || (int)gl + dir >= G;
+    // the neighbouring register (compile-time indices: no local-memory array)
+    const uint4 o = dir > 0 ? a[r + 1 < R ? r + 1 : R - 1] : a[r > 0 ? r - 1 : 0];
+    uint4 x, y;
+    x.x = __shfl_sync(gmask, a[r].x, src, G);
+    x.y = __shfl_sync(gmask, a[r].y, src, G);
+    x.z = __shfl_sync(gmask, a[r].z, src, G);
+    x.w = __shfl_sync(gmask, a[r].w, src, G);
+    if (R > 1) {
+        y.x = __shfl_sync(gmask, o.x, src, G);
+        y.y = __shfl_sync(gmask, o.y, src, G);
+        y.z = __shfl_sync(gmask, o.z, src, G);
+        y.w = __shfl_sync(gmask, o.w, src, G);
+        if (wrap) x = y;
+    }
+    return x;
+}
+__device__ __forceinline__ uint32_t w4(const uint4 &v, int k) {
+    return k == 0 ? v.x : (k == 1 ? v.y : (k == 2 ? v.z : v.w));
+}
+// Words k of the shifted vector: out[k] = cat(lo, hi)[k + s], s in 0..3.
+__device__ __forceinline__ uint4 funnel4(const uint4 &lo, const uint4 &hi, int s) {
+    switch (s) {
+        case 0: return lo;
+        case 1: return make_uint4(lo.y, lo.z, lo.w, hi.x);
+        case 2: return make_uint4(lo.z, lo.w, hi.x, hi.y);
+        default: return make_uint4(lo.w, hi.x, hi.y, hi.z);
+    }
+}
+
+struct SegUaParams {
+    char *base;
+    uint64_t ostride, istride;   // bytes between outer / inner batch items
+    uint64_t S;                  // unit bytes (multiple of 4)
+    uint64_t A;
+    FastDiv divB, divInner, divNch, divNseg;
+    uint64_t nch;                // chunks per unit
+    uint32_t cw;                 // words per (full) chunk, multiple of 4
+    uint32_t nw;                 // words per unit
+    const ulonglong2 *segs;
+    uint64_t nseg, tasks;
+    unsigned int *bar;
+    int self_reset;
+    uint32_t zero;
+};
+
+template <int G, int R>
+__global__ void __launch_bounds__(256, 4) cycle_seg_ua_kernel(const SegUaParams p) {
+    const uint32_t gl = threadIdx.x % G;
+    const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << ((threadIdx.x & 31) - gl));
+    const uint64_t w = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) / G;
+    const bool act = w < p.tasks;
+    uint4 D[R], Bk[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) D[r] = Bk[r] = make_uint4(0, 0, 0, 0);
+    char *ib = nullptr;
+    uint64_t cur = 0, len = 0, coff = 0;   // coff: byte offset of the chunk in its unit
+    uint32_t nwc = 0;                      // words in this chunk
+    int o = 0;                             // word phase of the carried chunk
+    if (act) {
+        uint64_t rest, ch, item, seg, to, ti;
+        fdivmod(w, p.divNch, rest, ch);
+        fdivmod(rest, p.divNseg, item, seg);
+        fdivmod(item, p.divInner, to, ti);
+        ib = p.base + to * p.ostride + ti * p.istride;
+        const ulonglong2 sg = p.segs[seg];
+        cur = sg.x;
+        len = sg.y;
+        coff = ch * (uint64_t)p.cw * 4;
+        nwc = (uint32_t)min((uint64_t)p.cw, (uint64_t)p.nw - ch * p.cw);
+        const uintptr_t a = (uintptr_t)(ib + cur * p.S + coff);
+        o = (int)((a & 15) >> 2);
+        const char *vb = (const char *)(a & ~(uintptr_t)15);
+        const uint32_t nvv = (o + nwc + 3) >> 2;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const uint32_t v = r * G + gl;
+            if (v < nvv) D[r] = ld_cg<16>(vb + (size_t)v * 16);
+        }
+    }
+    uint32_t f = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) f |= fold(D[r]);
+    if ((f & p.zero) != 0) __trap();
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+        atomicAdd(p.bar, 1u);
+        uint32_t seen = 0;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(seen) : "l"(p.bar) : "memory");
+        } while (seen < gridDim.x);
+        if (p.self_reset && atomicAdd(p.bar + 1, 1u) == gridDim.x - 1) {
+            atomicExch(p.bar, 0u);
+            atomicExch(p.bar + 1, 0u);
+        }
+    }
+    __syncthreads();
+    if (!act) return;   // whole walkers: a group's lanes share one task
+    for (uint64_t i = 1; i <= len; ++i) {
+        uint64_t q, rr;
+        fdivmod(cur, p.divB, q, rr);
+        const uint64_t d = rr * p.A + q;             // Eq. (1) on units
+        const uintptr_t a = (uintptr_t)(ib + d * p.S + coff);
+        const int pt = (int)((a & 15) >> 2);         // target phase
+        char *vb = (char *)(a & ~(uintptr_t)15);
+        const uint32_t nvt = (pt + nwc + 3) >> 2;    // covering vectors of the target
+        uint32_t z = 0;
+        if (i < len) {
+#pragma unroll
+            for (int r = 0; r < R; ++r) {
+                const uint32_t v = r * G + gl;
+                if (v < nvt) Bk[r] = ld_cg<16>(vb + (size_t)v * 16);
+            }
+            uint32_t f2 = 0;   // stores wait for the backup (see cycle_seg_kernel)
+#pragma unroll
+            for (int r = 0; r < R; ++r) f2 |= fold(Bk[r]);
+            z = f2 & p.zero;
+        }
+        vb += z;
+        // target vector v, word k = carried chunk word (4v + k - pt) = carried covering word
+        // (4v + k - dsh), dsh = pt - o: from vectors (v, v+1) at shift -dsh, or (v-1, v) at
+        // shift 4 - dsh
+        const int dsh = pt - o;
+        const int dir = dsh <= 0 ? 1 : -1;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const uint4 nb = group_vec_nb<G, R>(D, r, gl, dir, gmask);
+            const uint4 outv = dsh <= 0 ? funnel4(D[r], nb, -dsh) : funnel4(nb, D[r], 4 - dsh);
+            const uint32_t v = r * G + gl;
+            if (v < nvt) {
+                const int t0 = (int)(4 * v) - pt;      // chunk word held by component 0
+                char *dst = vb + (size_t)v * 16;
+                if (t0 >= 0 && t0 + 3 < (int)nwc) {
+                    st_cg<16>(dst, outv);
+                } else {
+#pragma unroll
+                    for (int k = 0; k < 4; ++k)
+                        if (t0 + k >= 0 && t0 + k < (int)nwc) st_cg<4>(dst + 4 * k, w4(outv, k));
+                }
+            }
+        }
+        if (i < len) {
+#pragma unroll
+            for (int r = 0; r < R; ++r) D[r] = Bk[r];
+            o = pt;
+        }
+        cur = d;
+    }
+}
+
 // ------------------------------------------------------------------------ host side
 namespace {
 
@@ -204,9 +371,48 @@ bool build_segments(uint64_t A, uint64_t B, uint64_t max_seg, std::vector<ulongl
 struct SegCfg {
     int G, R;
     uint64_t nch, chunk;
+    bool ua = false;     // unaligned units: cycle_seg_ua_kernel, chunk = cw words
+    uint32_t cw = 0;
 };
 
-SegCfg seg_cfg(uint64_t S) {
+// Unaligned units: a walker of G lanes x R vectors covers cap = G*R vectors; a chunk of cw
+// words covers at most (cw + 6) / 4 of them at any phase, so cw + 3 <= 4 cap.  One chunk per
+// unit with the smallest cap (ties: fewest lanes, i.e. most walkers per warp) up to 508
+// words; beyond, greedy 508-word (2032-byte) chunks on 32 x 4 walkers.
+SegCfg seg_cfg_ua(uint64_t S) {
+    const uint64_t nw = S / 4;
+    SegCfg c{32, 4, 1, 0, true, 0};
+    uint64_t best = ~0ull;
+    const long gmin = env_int("IPT_SEG_UA_G", 8);   // smallest walker width considered
+    for (int G : {8, 16, 32})
+        if (G >= gmin)
+        for (int R = 1; R <= 4; R *= 2) {
+            const uint64_t cap = (uint64_t)G * R;
+            if (nw + 3 <= 4 * cap && cap < best) {
+                best = cap;
+                c.G = G;
+                c.R = R;
+                c.cw = (uint32_t)((nw + 3) & ~3ull);
+            }
+        }
+    if (!c.cw) {
+        c.G = 32;
+        c.R = 4;
+        c.cw = 508;
+        c.nch = (nw + 507) / 508;
+    }
+    c.chunk = (uint64_t)c.cw * 4;
+    return c;
+}
+
+// Is a stage with S-byte units run by the unaligned kernel?  (S % 16 != 0, or data not
+// 16-byte aligned; 4-byte granular units only.)
+bool seg_unaligned(uint64_t S, uintptr_t base, bool strided, uint64_t ostride) {
+    return S % 16 || (base & 15) || (strided && (ostride & 15));
+}
+
+SegCfg seg_cfg(uint64_t S, bool ua = false) {
+    if (ua || S % 16) return seg_cfg_ua(S);
     const uint64_t nv = S / 16;
     static const int Gs[3] = {8, 16, 32};
     SegCfg best{32, 4, (nv + 127) / 128, 32 * 4 * 16};
@@ -235,7 +441,14 @@ SegCfg seg_cfg(uint64_t S) {
 template <int G, int R>
 void *seg_kernel_ptr() { return (void *)cycle_seg_kernel<G, R>; }
 
-void *seg_kernel(int G, int R) {
+void *seg_kernel(int G, int R, bool ua = false) {
+    if (ua) {
+#define IPT_SEG_UA(g, r) if (G == g && R == r) return (void *)cycle_seg_ua_kernel<g, r>;
+        IPT_SEG_UA(8, 1) IPT_SEG_UA(8, 2) IPT_SEG_UA(8, 4) IPT_SEG_UA(16, 1) IPT_SEG_UA(16, 2)
+        IPT_SEG_UA(16, 4) IPT_SEG_UA(32, 1) IPT_SEG_UA(32, 2) IPT_SEG_UA(32, 4)
+#undef IPT_SEG_UA
+        return nullptr;
+    }
 #define IPT_SEG_K(g, r) if (G == g && R == r) return seg_kernel_ptr<g, r>();
     IPT_SEG_K(8, 1) IPT_SEG_K(8, 2) IPT_SEG_K(8, 3) IPT_SEG_K(8, 4)
     IPT_SEG_K(16, 1) IPT_SEG_K(16, 2) IPT_SEG_K(16, 3) IPT_SEG_K(16, 4)
@@ -350,9 +563,9 @@ bool seg_plan_ready(SegPlan &sp, cudaStream_t st, bool capturing) {
 
 // Walkers a launch can keep co-resident for a stage with S-byte units (0: not applicable).
 uint64_t cycle_seg_walkers(int64_t S_bytes, int device) {
-    if (S_bytes % 16) return 0;
+    if (S_bytes % 4 || (S_bytes % 16 && !env_int("IPT_SEG_UA", 1))) return 0;
     const SegCfg c = seg_cfg((uint64_t)S_bytes);
-    void *k = seg_kernel(c.G, c.R);
+    void *k = seg_kernel(c.G, c.R, c.ua);
     const int per_sm = device >= 0 ? seg_blocks_per_sm(k) : 4;
     return (uint64_t)dev_props(device).sms * per_sm * 256 / c.G;
 }
@@ -361,12 +574,17 @@ uint64_t cycle_seg_walkers(int64_t S_bytes, int device) {
 // flag kernel is used instead.
 constexpr uint64_t kSegMaxUnits = 1ull << 26;
 
+bool stage_unaligned(const StageDesc &d) {
+    return seg_unaligned((uint64_t)(d.s * d.eb), (uintptr_t)d.base, d.outer > 1, (uint64_t)d.ostride);
+}
+
 bool cycle_seg_applicable(const StageDesc &d) {
     const uint64_t S = (uint64_t)(d.s * d.eb);
-    if (S % 16 || ((uintptr_t)d.base & 15)) return false;
     if ((uint64_t)(d.A * d.B) > kSegMaxUnits) return false;
-    if (d.outer > 1 && (d.ostride & 15)) return false;
-    return true;
+    if (!stage_unaligned(d)) return true;
+    // unaligned units: 4-byte granular (the walker moves whole words)
+    if (S % 4 || ((uintptr_t)d.base & 3) || (d.outer > 1 && (d.ostride & 3))) return false;
+    return env_int("IPT_SEG_UA", 1) != 0;
 }
 
 size_t cycle_seg_ws_bytes() { return 256; }
@@ -376,8 +594,9 @@ size_t cycle_seg_ws_bytes() { return 256; }
 cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int device) {
     if (!cycle_seg_applicable(d)) return cudaErrorNotSupported;
     const uint64_t S = (uint64_t)(d.s * d.eb);
-    const SegCfg c = seg_cfg(S);
-    void *k = seg_kernel(c.G, c.R);
+    const bool ua = stage_unaligned(d);
+    const SegCfg c = seg_cfg(S, ua);
+    void *k = seg_kernel(c.G, c.R, ua);
     const int per_sm = seg_blocks_per_sm(k);
     if (per_sm < 1) return cudaErrorNotSupported;
     const uint64_t items = (uint64_t)(d.outer * d.inner);
@@ -394,6 +613,48 @@ cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int 
     if (!sp->ok) return cudaErrorNotSupported;
     if (sp->nseg == 0) return cudaSuccess;   // identity permutation
     if (!seg_plan_ready(*sp, st, cap != cudaStreamCaptureStatusNone)) return cudaErrorNotSupported;
+    unsigned int *ctr = nullptr;
+    if (env_int("IPT_SEG_RESET", 1))
+        ctr = cap == cudaStreamCaptureStatusNone ? seg_counters(device, st) : nullptr;   // captured: workspace
+    if (!ctr) {
+        const cudaError_t e = cudaMemsetAsync(ws, 0, 2 * sizeof(unsigned int), st);
+        if (e != cudaSuccess) return e;
+    }
+    if (ua) {
+        SegUaParams u{};
+        u.base = d.base;
+        u.ostride = (uint64_t)d.ostride;
+        u.istride = (uint64_t)(d.A * d.B) * S;
+        u.S = S;
+        u.A = (uint64_t)d.A;
+        u.divB = make_fastdiv((uint64_t)d.B);
+        u.divInner = make_fastdiv((uint64_t)d.inner);
+        u.divNch = make_fastdiv(c.nch);
+        u.divNseg = make_fastdiv(sp->nseg);
+        u.nch = c.nch;
+        u.cw = c.cw;
+        u.nw = (uint32_t)(S / 4);
+        u.segs = (const ulonglong2 *)sp->dev;
+        u.nseg = sp->nseg;
+        u.tasks = items * sp->nseg * c.nch;
+        u.bar = ctr ? ctr : (unsigned int *)ws;
+        u.self_reset = ctr ? 1 : 0;
+        u.zero = 0;
+        const uint64_t blocks_needed = (u.tasks * c.G + 255) / 256;
+        const unsigned grid = (unsigned)std::min<uint64_t>(blocks_needed, (uint64_t)dev_props(device).sms * per_sm);
+        if (env_int("IPT_DEBUG", 0))
+            fprintf(stderr, "[ipt] cycle_seg_ua A=%lld B=%lld S=%llu G=%d R=%d cw=%u nch=%llu L=%llu nseg=%llu grid=%u\n",
+                    (long long)d.A, (long long)d.B, (unsigned long long)S, c.G, c.R, c.cw,
+                    (unsigned long long)c.nch, (unsigned long long)sp->L, (unsigned long long)sp->nseg, grid);
+        void *args[] = {&u};
+        cudaError_t e = cudaLaunchCooperativeKernel(k, dim3(grid), dim3(256), args, 0, st);
+        if (e == cudaErrorCooperativeLaunchTooLarge || e == cudaErrorNotSupported) {
+            cudaGetLastError();
+            return cudaErrorNotSupported;
+        }
+        note_launch();
+        return e != cudaSuccess ? e : cudaGetLastError();
+    }
     SegParams p{};
     p.base = d.base;
     p.ostride = (uint64_t)d.ostride;
@@ -414,20 +675,10 @@ cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int 
     p.diag = (int)env_int("IPT_SEG_DIAG", 0);
     // barrier counters: a library-owned, self-resetting pair per (device, stream) -- no memset
     // node per launch (2 us of a ~40 us configs[0] transposition); the caller's workspace
-    // with a memset when the pair cannot be created (e.g. first use inside stream capture)
-    unsigned int *ctr = nullptr;
-    if (env_int("IPT_SEG_RESET", 1))
-        ctr = cap == cudaStreamCaptureStatusNone ? seg_counters(device, st) : nullptr;   // captured: workspace
+    // with a memset (above) when the pair cannot be used (stream capture, IPT_SEG_RESET=0)
     cudaError_t e = cudaSuccess;
-    if (ctr) {
-        p.bar = ctr;
-        p.self_reset = 1;
-    } else {
-        p.bar = (unsigned int *)ws;
-        p.self_reset = 0;
-        e = cudaMemsetAsync(ws, 0, 2 * sizeof(unsigned int), st);
-        if (e != cudaSuccess) return e;
-    }
+    p.bar = ctr ? ctr : (unsigned int *)ws;
+    p.self_reset = ctr ? 1 : 0;
     const uint64_t blocks_needed = (p.tasks * c.G + 255) / 256;
     const unsigned grid = (unsigned)std::min<uint64_t>(blocks_needed, (uint64_t)dev_props(device).sms * per_sm);
     if (env_int("IPT_DEBUG", 0))
@@ -445,13 +696,16 @@ cudaError_t launch_cycle_seg(const StageDesc &d, void *ws, cudaStream_t st, int 
     return e != cudaSuccess ? e : cudaGetLastError();
 }
 
+const char *cycle_seg_name(const StageDesc &d) { return stage_unaligned(d) ? "cycle_seg_ua" : "cycle_seg"; }
+
 // Would launch_cycle_seg run this stage (diagnostics)?  Without a cached segment plan the
 // cycles are not walked here: a stage with more cycles than walkers (rare) is reported as
 // segmented although the launcher then falls back to the flag kernel.
 bool cycle_seg_would_launch(const StageDesc &d, int device) {
     if (!cycle_seg_applicable(d)) return false;
-    const SegCfg c = seg_cfg((uint64_t)(d.s * d.eb));
-    const int per_sm = seg_blocks_per_sm(seg_kernel(c.G, c.R));
+    const bool ua = stage_unaligned(d);
+    const SegCfg c = seg_cfg((uint64_t)(d.s * d.eb), ua);
+    const int per_sm = seg_blocks_per_sm(seg_kernel(c.G, c.R, ua));
     if (per_sm < 1) return false;
     const uint64_t items = (uint64_t)(d.outer * d.inner);
     const uint64_t walkers = (uint64_t)dev_props(device).sms * per_sm * 256 / c.G;

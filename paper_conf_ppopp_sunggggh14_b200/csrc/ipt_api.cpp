@@ -17,6 +17,7 @@
 #include <cstring>
 #include <map>
 #include <mutex>
+#include <string>
 #include <vector>
 
 namespace ipt {
@@ -30,13 +31,71 @@ void fill_plan(int64_t M, int64_t N, int64_t m, int64_t n, int eb, int device, i
 static std::atomic<uint64_t> g_launches{0};
 void note_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
 
-long env_int(const char *name, long dflt) {
-    const char *v = std::getenv(name);
-    if (!v || !*v) return dflt;
-    char *end = nullptr;
-    long x = std::strtol(v, &end, 10);
-    return (end && *end == 0) ? x : dflt;
+// Tuning knobs (IPT_* environment variables; tests and measurements only).  The launch
+// path reads dozens of them per stage, so instead of a getenv (a scan of the whole
+// environment) per read, the IPT_* entries are snapshot once per thread and re-scanned
+// only when the environment block changes (environ pointer, entry count or the IPT_*
+// strings -- what setenv/putenv, and so Python's os.environ, modify).
+extern "C" char **environ;
+
+namespace {
+struct EnvSnap {
+    char **env = nullptr;
+    size_t count = 0;
+    uint64_t hash = 0;
+    std::vector<std::pair<std::string, std::string>> kv;
+};
+thread_local EnvSnap g_env;
+
+void env_scan(EnvSnap &s) {
+    s.env = environ;
+    s.count = 0;
+    s.kv.clear();
+    uint64_t h = 1469598103934665603ull;
+    for (char **e = environ; e && *e; ++e) {
+        ++s.count;
+        if (std::strncmp(*e, "IPT_", 4) != 0) continue;
+        const char *eq = std::strchr(*e, '=');
+        if (!eq) continue;
+        s.kv.emplace_back(std::string(*e, eq - *e), std::string(eq + 1));
+        for (const char *c = *e; *c; ++c) h = (h ^ (uint8_t)*c) * 1099511628211ull;
+    }
+    s.hash = h;
 }
+
+// Cheap check that the snapshot is current: same environ block and entry count, and each
+// recorded IPT_* value still the same (getenv only for the few IPT_* names present).
+const EnvSnap &env_now() {
+    EnvSnap &s = g_env;
+    bool fresh = s.env == environ && s.env != nullptr;
+    if (fresh) {
+        size_t n = 0;
+        for (char **e = environ; *e; ++e) ++n;
+        fresh = n == s.count;
+        for (size_t i = 0; fresh && i < s.kv.size(); ++i) {
+            const char *v = std::getenv(s.kv[i].first.c_str());
+            fresh = v && s.kv[i].second == v;
+        }
+    }
+    if (!fresh) env_scan(s);
+    return s;
+}
+}  // namespace
+
+long env_int(const char *name, long dflt) {
+    const EnvSnap &s = env_now();
+    for (const auto &kv : s.kv) {
+        if (kv.first != name) continue;
+        const char *v = kv.second.c_str();
+        if (!*v) return dflt;
+        char *end = nullptr;
+        long x = std::strtol(v, &end, 10);
+        return (end && *end == 0) ? x : dflt;
+    }
+    return dflt;
+}
+
+uint64_t env_hash() { return env_now().hash; }
 
 FastDiv make_fastdiv(uint64_t d) {
     FastDiv f{};

@@ -99,11 +99,13 @@ bool tile_onchip_fits(int64_t A, int64_t B, int eb, int device);
 // 3: 16-byte path split over a thread-block cluster (tile_cluster_k CTAs),
 // 4: element path split over a thread-block cluster,
 // 5: 16-byte path split over a co-resident group of CTAs (double-buffered slices),
-// 6: element path (4/8-byte elements) split over a co-resident group of CTAs
+// 6: element path (4/8-byte elements) split over a co-resident group of CTAs,
+// 7: 16-byte path over every SM, slices in shared memory + registers (tile_group_rf)
 int tile_onchip_path(int64_t A, int64_t B, int eb, int device);
 int tile_cluster_k(int64_t A, int64_t B, int eb, int device);
 int tile_generic_cluster_k(int64_t A, int64_t B, int eb, int device);
 bool tile_group_split(int64_t A, int64_t B, int eb, int device);
+bool tile_rf_fits(int64_t A, int64_t B, int eb, int device);   // whole-GPU smem + register tiles
 bool tile_group_generic_split(int64_t A, int64_t B, int eb, int device);
 // Group split of `count` tiles: CTAs per tile (0 = does not fit) and groups in flight.
 int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *groups,
@@ -140,5 +142,6 @@ void note_launch();
 
 // Environment-variable integer override (tuning knobs for tests / sweeps).
 long env_int(const char *name, long dflt);
+uint64_t env_hash();   // hash of the IPT_* variables set (cache keys of env-dependent plans)
 
 }  // namespace ipt

@@ -34,6 +34,7 @@
 #include <cstdio>
 #include <map>
 #include <mutex>
+#include <tuple>
 
 namespace ipt {
 
@@ -69,6 +70,8 @@ struct TileParams {
                           // to a second buffer after the data; 16 = timeline
                           // trace (results valid, see ipt__tile_trace)
     unsigned long long *trace;
+    uint32_t rows_a;      // tile_group_rf: slice rows staged in shared memory by TMA (rest: registers)
+    uint32_t zero;        // 0 at run time, opaque to the compiler (load-completion dependency)
 };
 
 __device__ __forceinline__ char *tile_ptr(const TileParams &p, uint64_t t) {
@@ -688,6 +691,166 @@ __global__ void __launch_bounds__(512, 1) tile_group_tma(const TileParams p, con
         [&](char *g, uint32_t sb, auto probe) {
             write_out_pan<EB>(p, sb, g, q, divq, pstride, b0, nb, divnb, c0, cvec, probe);
         });
+}
+
+// ------------------- whole-GPU tiles held in shared memory AND tensor memory (rf)
+// Tiles too large even for single-buffered slices over every SM (e.g. one 4096 x 3000 or
+// 1800 x 7200 float32 matrix, 49-52 MB, as ONE tile: the plan m = M, n = N, stages 1 and 3
+// identities -- P:315's "tile fits on chip" taken to the whole B200).  The aggregate
+// on-chip storage of 148 SMs is shared memory (148 x 227 KB) plus Blackwell's tensor memory
+// (TMEM, 148 x 256 KB, otherwise the MMA accumulator store; here plain staging).  A group of
+// K CTAs (one per SM, 512 threads) owns a tile; CTA k's slice (row or column split, as
+// tile_group_tma) is held as
+//   part A: its first rows_a rows, fetched by 2-D TMA boxes into the column-panel layout;
+//   part B: the remaining rows, loaded by the threads with 16-byte loads (consecutive
+//           threads, consecutive vectors of a row) and parked in TMEM with tcgen05.st --
+//           each thread owns 128 columns of its warp's lane quarter (512 B, RV <= 32
+//           vectors), so no register is held across the write-out.
+// In-place rule as the group kernels: the CTA arrives on the group counter once part A has
+// landed (mbarrier) and every part-B load has returned (its value was stored to TMEM), and
+// no CTA stores into the tile before all K arrived.  Write-out: part A from shared memory
+// (write_out_pan: transposed V x V register blocks, coalesced 16-byte stores), then part B
+// is brought back (tcgen05.ld), stored into the freed shared memory in the same panel layout
+// and written out the same way.  Tiles of a group run one after another (a batch: the
+// spread of the CTAs overlaps one tile's stores with the next tile's loads across the GPU).
+__device__ __forceinline__ void tm_st4(uint32_t taddr, const uint4 &v) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1, %2, %3, %4};"
+                 :: "r"(taddr), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+__device__ __forceinline__ uint4 tm_ld4(uint32_t taddr) {
+    uint4 v;
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(taddr) : "memory");
+    return v;
+}
+
+constexpr int kRfBatch = 8;   // part-B vectors per thread in registers at a time
+
+template <int EB, int RV>
+__global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, const __grid_constant__ CUtensorMap tmap) {
+    constexpr int V = 16 / EB;
+    static_assert(RV % kRfBatch == 0 && RV <= 32, "TMEM holds 32 vectors per thread");
+    extern __shared__ __align__(128) unsigned char smem[];
+    const uint32_t s0 = smem_u32(smem);
+    const uint32_t K = p.K, rank = blockIdx.x % K, gid = blockIdx.x / K, ng = gridDim.x / K;
+    const uint32_t warp = threadIdx.x >> 5;
+    const uint32_t mv = p.m / V, nvr = p.n / V;
+    uint32_t b0, b1, c0, c1;
+    if (!p.colsplit) {
+        b0 = (uint32_t)((uint64_t)rank * mv / K);
+        b1 = (uint32_t)((uint64_t)(rank + 1) * mv / K);
+        c0 = 0; c1 = nvr;
+    } else {
+        b0 = 0; b1 = mv;
+        c0 = (uint32_t)((uint64_t)rank * nvr / K);
+        c1 = (uint32_t)((uint64_t)(rank + 1) * nvr / K);
+    }
+    const uint32_t q = p.q, cvec = c1 - c0;
+    const uint32_t rows = (b1 - b0) * V, r0 = b0 * V;
+    const uint32_t ra = min(p.rows_a, rows), rb = rows - ra;        // rows in smem / TMEM
+    const uint32_t nvb = rb * cvec;                                    // part-B vectors of the slice
+    const uint32_t pstride_b = ((rb * q * 16) + 127) & ~127u;
+    const FastDiv32 divq = make_fastdiv32_dev(q), divc = make_fastdiv32_dev(cvec);
+    const FastDiv32 diva = make_fastdiv32_dev(ra / V), divb = make_fastdiv32_dev(rb / V);
+    __shared__ __align__(8) uint64_t mbar;
+    __shared__ uint32_t tmem_base;
+    if (warp == 0) {   // all 512 TMEM columns of this SM (one CTA per SM)
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;"
+                     :: "r"(smem_u32(&tmem_base)) : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
+    if (threadIdx.x == 0) {
+        mbar_init(&mbar, 1);
+        fence_mbar_init();
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    // this thread's 128 columns in its warp's lane quarter
+    const uint32_t taddr = tmem_base + ((32u * (warp & 3)) << 16) + (warp >> 2) * 128u;
+    uint32_t *ctr = p.gbar + gid * (kGroupCtrStride / 4);
+    const uint32_t nt = gid < p.count ? (uint32_t)((p.count - gid + ng - 1) / ng) : 0;
+    for (uint32_t i = 0; i < nt; ++i) {
+        char *g = tile_ptr(p, gid + (uint64_t)i * ng);
+        // ---- part A: TMA boxes (rows_a rows of every panel; boxes may read past the slice)
+        if (threadIdx.x == 0) {
+            const uint64_t row0 = (uint64_t)(g - p.base) / ((uint64_t)p.n * EB) + r0;
+            mbar_arrive_expect_tx(&mbar, p.npan * p.rows_a * q * 16);
+            const uint32_t sbar = smem_u32(&mbar);
+            for (uint32_t pn = 0; pn < p.npan; ++pn)
+                for (uint32_t r = 0; r < p.rows_a; r += p.box_rows)
+                    tma_load_2d(s0 + pn * p.pstride + r * q * 16, &tmap, (int32_t)((c0 + pn * q) * V),
+                                (int32_t)(row0 + r), sbar);
+        }
+        // ---- part B: 16-byte loads, parked in TMEM batch by batch
+        const char *gb = g + ((size_t)(r0 + ra) * nvr + c0) * 16;
+        if (!(p.diag & 4)) {
+#pragma unroll 1
+            for (int u0 = 0; u0 < RV; u0 += kRfBatch) {
+                if ((uint32_t)u0 * 512 >= nvb) break;
+                uint4 v[kRfBatch];
+#pragma unroll
+                for (int j = 0; j < kRfBatch; ++j) {
+                    const uint32_t e = threadIdx.x + (uint32_t)(u0 + j) * 512;
+                    v[j] = make_uint4(0, 0, 0, 0);
+                    if (e < nvb) {
+                        uint32_t r, c;
+                        fdivmod32(e, divc, r, c);
+                        v[j] = ld_cg<16>(gb + ((size_t)r * nvr + c) * 16);
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < kRfBatch; ++j) tm_st4(taddr + 4u * (uint32_t)(u0 + j), v[j]);
+            }
+            asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        }
+        mbar_wait(&mbar, i & 1);            // part A has landed
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            group_arrive(ctr, p.arrive_release != 0);
+            if (!(p.diag & 1)) group_wait(ctr, K * (i + 1));   // all slices of the tile on chip
+        }
+        __syncthreads();
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        // ---- write-out: part A, then part B through the freed shared memory
+        if (ra && !(p.diag & 2))
+            write_out_pan<EB>(p, s0, g, q, divq, p.pstride, r0 / V, ra / V, diva, c0, cvec, NoProbe());
+        __syncthreads();
+#pragma unroll 1
+        for (int u0 = 0; u0 < RV; u0 += kRfBatch) {
+            if ((uint32_t)u0 * 512 >= nvb) break;
+            uint4 v[kRfBatch];
+#pragma unroll
+            for (int j = 0; j < kRfBatch; ++j) v[j] = tm_ld4(taddr + 4u * (uint32_t)(u0 + j));
+            asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+            for (int j = 0; j < kRfBatch; ++j) {
+                const uint32_t e = threadIdx.x + (uint32_t)(u0 + j) * 512;
+                if (e < nvb) {
+                    uint32_t r, c, pn, pc;
+                    fdivmod32(e, divc, r, c);
+                    fdivmod32(c, divq, pn, pc);
+                    sts128(s0 + pn * pstride_b + (r * q + pc) * 16, v[j]);
+                }
+            }
+        }
+        __syncthreads();
+        if (rb && !(p.diag & 2))
+            write_out_pan<EB>(p, s0, g, q, divq, pstride_b, (r0 + ra) / V, rb / V, divb, c0, cvec, NoProbe());
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        __syncthreads();
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    }
+    if (warp == 0)
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tmem_base) : "memory");
+    if (p.gexit && threadIdx.x == 0) {   // self-resetting counters (see group_loop)
+        uint32_t *ex = p.gexit + gid * (kGroupCtrStride / 4);
+        if (atomicAdd(ex, 1u) == K - 1) {
+            atomicExch(ctr, 0u);
+            atomicExch(ex, 0u);
+        }
+    }
 }
 
 // --------------------------------- group-split element path with TMA slices (aligned rows)
@@ -1379,7 +1542,26 @@ static GroupCfg group_search_nb(int64_t A, int64_t B, int eb, uint64_t count, in
     return g;
 }
 
+static GroupCfg group_choose_uncached(int64_t A, int64_t B, int eb, uint64_t count, int device, bool generic);
+
+// Group configurations are searched over every K (and both split directions): cached per
+// (shape, count, device, IPT_* knobs) so that a launch or a plan evaluation costs a lookup.
 static GroupCfg group_choose(int64_t A, int64_t B, int eb, uint64_t count, int device, bool generic) {
+    static std::mutex mu;
+    static std::map<std::tuple<int64_t, int64_t, int, uint64_t, int, bool, uint64_t>, GroupCfg> cache;
+    const auto key = std::make_tuple(A, B, eb, count, device, generic, env_hash());
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = cache.find(key);
+        if (it != cache.end()) return it->second;
+    }
+    const GroupCfg g = group_choose_uncached(A, B, eb, count, device, generic);
+    std::lock_guard<std::mutex> lk(mu);
+    cache[key] = g;
+    return g;
+}
+
+static GroupCfg group_choose_uncached(int64_t A, int64_t B, int eb, uint64_t count, int device, bool generic) {
     const long f = env_int("IPT_TILE_GROUP_COLSPLIT", -1);
     if (f >= 0) return group_search(A, B, eb, count, device, f != 0, generic);
     const GroupCfg row = group_search(A, B, eb, count, device, false, generic);
@@ -1614,6 +1796,153 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
     return e != cudaSuccess ? e : cudaGetLastError();
 }
 
+// Whole-GPU tiles in shared memory + registers (tile_group_rf): K = every SM, one group.
+struct RfCfg {
+    int K = 0, rv = 0;
+    bool colsplit = false;
+    uint32_t q = 0, npan = 0, rows_a = 0, box_rows = 0;
+    size_t pstride = 0, smem = 0;
+};
+constexpr int kRfThreads = 512;
+constexpr int kRfMaxRV = 32;   // part-B vectors per thread in TMEM (128 columns x 4 B)
+
+static RfCfg rf_search(int64_t A, int64_t B, int eb, int device, bool cs) {
+    RfCfg c;
+    const DevProps dp = dev_props(device);
+    const int K = dp.sms, V = 16 / eb;
+    const int64_t mv = A / V, nvr = B / V;
+    if ((cs ? nvr : mv) < K) return c;
+    const int64_t rows = cs ? A : (mv + K - 1) / K * V;                 // max slice rows
+    const int64_t cvec = cs ? (nvr + K - 1) / K : nvr;                   // max slice vectors per row
+    const uint32_t maxw = 256 / V - 1;
+    const uint32_t npan = (uint32_t)((cvec + maxw - 1) / maxw);
+    const uint32_t q = (uint32_t)(((cvec + npan - 1) / npan) | 1);
+    const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin) - 1024;
+    auto pst = [&](int64_t r) { return (size_t)((r * q * 16 + 127) & ~(int64_t)127); };
+    for (int64_t ra = rows / V * V; ra >= V; ra -= V) {
+        if ((long)(npan * pst(ra)) > budget) continue;
+        uint32_t br = 0;                                   // TMA box rows (128-B aligned boxes)
+        if (ra <= 256) br = (uint32_t)ra;
+        else
+            for (uint32_t b = 256; b >= 16; b -= 8)
+                if (ra % b == 0) { br = b; break; }
+        if (!br) continue;
+        const int64_t rb = rows - ra;
+        const int64_t rv = (rb * cvec + kRfThreads - 1) / kRfThreads;
+        if (rv > kRfMaxRV || (long)(npan * pst(rb)) > budget) return c;   // fewer rows in smem only adds registers
+        c.K = K;
+        c.colsplit = cs;
+        c.q = q;
+        c.npan = npan;
+        c.rows_a = (uint32_t)ra;
+        c.box_rows = br;
+        c.rv = (int)rv;
+        c.pstride = pst(ra);
+        c.smem = std::max(npan * pst(ra), npan * pst(rb));
+        return c;
+    }
+    return c;
+}
+
+static RfCfg rf_cfg(int64_t A, int64_t B, int eb, int device) {
+    if ((eb != 4 && eb != 8) || !vec_ok(A, B, eb) || !env_int("IPT_TILE_RF", 1)) return RfCfg{};
+    static std::mutex mu;
+    static std::map<std::tuple<int64_t, int64_t, int, int, uint64_t>, RfCfg> cache;
+    const auto key = std::make_tuple(A, B, eb, device, env_hash());
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = cache.find(key);
+        if (it != cache.end()) return it->second;
+    }
+    const int K = dev_props(device).sms;
+    const bool row_first = A * eb / K >= 64;   // as group_choose: row-split pieces >= 64 B
+    RfCfg c = rf_search(A, B, eb, device, !row_first);
+    if (!c.K) c = rf_search(A, B, eb, device, row_first);
+    std::lock_guard<std::mutex> lk(mu);
+    cache[key] = c;
+    return c;
+}
+
+template <int EB>
+cudaError_t launch_group_rf(const StageDesc &d, TileParams p, const RfCfg &c, void *ws, cudaStream_t st,
+                            int device) {
+    if (!ws || !c.K) return cudaErrorInvalidValue;
+    if (d.outer > 1 && d.ostride != d.inner * (int64_t)p.tile_bytes) return cudaErrorNotSupported;
+    auto enc = tensor_map_encoder();
+    if (!enc) return cudaErrorNotSupported;
+    const int V = 16 / EB;
+    CUtensorMap tm;
+    const uint64_t total_rows = (uint64_t)(d.outer * d.inner) * (uint64_t)d.A;
+    cuuint64_t dims[2] = {(cuuint64_t)d.B, (cuuint64_t)total_rows};
+    cuuint64_t strides[1] = {(cuuint64_t)(d.B * EB)};
+    cuuint32_t box[2] = {c.q * (uint32_t)V, c.box_rows};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(&tm, EB == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 2, d.base,
+                     dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return cudaErrorNotSupported;
+    p.q = c.q;
+    p.npan = c.npan;
+    p.pstride = (uint32_t)c.pstride;
+    p.box_rows = c.box_rows;
+    p.rows_a = c.rows_a;
+    p.colsplit = c.colsplit ? 1 : 0;
+    p.K = (uint32_t)c.K;
+    p.nbuf = 1;
+    p.zero = 0;
+    p.gbar = (uint32_t *)ws;
+    p.gexit = nullptr;
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(st, &cap) != cudaSuccess) { cudaGetLastError(); cap = cudaStreamCaptureStatusActive; }
+    if (env_int("IPT_TILE_RESET", 1) && cap == cudaStreamCaptureStatusNone) {
+        if (uint32_t *ctr = group_counters(device, st, true)) {
+            p.gbar = ctr;
+            p.gexit = ctr + kTileWsBytes / 4;
+        }
+    }
+    if (!p.gexit) {
+        const cudaError_t e = cudaMemsetAsync(ws, 0, kGroupCtrStride, st);
+        if (e != cudaSuccess) return e;
+    }
+    const void *kern = nullptr;
+    const int rv = (c.rv + kRfBatch - 1) / kRfBatch * kRfBatch;
+#define IPT_RF(R) if (rv == R) kern = (const void *)tile_group_rf<EB, R>;
+    IPT_RF(8) IPT_RF(16) IPT_RF(24) IPT_RF(32)
+#undef IPT_RF
+    if (!kern) return cudaErrorNotSupported;
+    {
+        static std::mutex mu;
+        static std::map<std::pair<const void *, int>, bool> done;
+        std::lock_guard<std::mutex> lk(mu);
+        if (!done[std::make_pair(kern, device)]) {
+            cudaFuncAttributes fa{};
+            cudaFuncGetAttributes(&fa, kern);
+            cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 dev_props(device).smem_optin - (int)fa.sharedSizeBytes);
+            done[std::make_pair(kern, device)] = true;
+        }
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)c.K, 1, 1);
+    cfg.blockDim = dim3(kRfThreads, 1, 1);
+    cfg.dynamicSmemBytes = c.smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    if (env_int("IPT_DEBUG", 0))
+        fprintf(stderr, "[ipt] tile_group_rf m=%u n=%u K=%d colsplit=%d q=%u npan=%u rows_a=%u box=%u rv=%d smem=%zu tiles=%llu\n",
+                p.m, p.n, c.K, p.colsplit, c.q, c.npan, c.rows_a, c.box_rows, rv, c.smem,
+                (unsigned long long)p.count);
+    void *args[] = {&p, &tm};
+    p.diag = (int)env_int("IPT_TILE_DIAG", 0);
+    cudaError_t e = cudaLaunchKernelExC(&cfg, kern, args);
+    note_launch();
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
+
 }  // namespace
 
 // Cluster size for a tile that does not fit one CTA (0 = none): the smallest K in
@@ -1731,8 +2060,12 @@ int tile_onchip_path(int64_t A, int64_t B, int eb, int device) {
     if (!vec_ok(A, B, eb) && tile_group_generic_split(A, B, eb, device)) return 6;
     if ((long)generic_smem(A, B, eb) > budget && tile_generic_cluster_k(A, B, eb, device)) return 4;
     if ((long)generic_smem(A, B, eb) <= budget && A * B < (1ll << 31)) return 1;
+    if (tile_rf_fits(A, B, eb, device)) return 7;
     return 0;
 }
+
+// A tile held over every SM in shared memory + registers (tile_group_rf)?
+bool tile_rf_fits(int64_t A, int64_t B, int eb, int device) { return rf_cfg(A, B, eb, device).K != 0; }
 
 // Name of the kernel launch_tile_onchip runs for this stage (diagnostics: the bench's
 // per-kernel roofline and the ncu launch lists use the same names).  Mirrors the launcher's
@@ -1765,6 +2098,9 @@ const char *tile_kernel_name(const StageDesc &d, int device) {
     }
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) > budget && tile_cluster_k(d.A, d.B, d.eb, device))
         return "tile_onchip_cluster";
+    if (fast_ok(d) && (d.eb == 4 || d.eb == 8) && (long)generic_smem(d.A, d.B, d.eb) > budget && packed &&
+        rf_cfg(d.A, d.B, d.eb, device).K)
+        return "tile_group_rf";
     if ((long)generic_smem(d.A, d.B, d.eb) > budget) return "tile_generic_cluster";
     return "tile_onchip_generic";
 }
@@ -1847,6 +2183,16 @@ cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, in
         switch (d.eb) {
             case 4: return launch_group_db<4, true>(d, p, g, ws, st, device);
             case 8: return launch_group_db<8, true>(d, p, g, ws, st, device);
+        }
+    }
+    if (fast_ok(d) && (d.eb == 4 || d.eb == 8) && !tile_cluster_k(d.A, d.B, d.eb, device) &&
+        (long)generic_smem(d.A, d.B, d.eb) > budget) {
+        const RfCfg c = rf_cfg(d.A, d.B, d.eb, device);
+        if (c.K) {
+            cudaError_t e = d.eb == 4 ? launch_group_rf<4>(d, p, c, ws, st, device)
+                                      : launch_group_rf<8>(d, p, c, ws, st, device);
+            if (e != cudaErrorNotSupported) return e;
+            cudaGetLastError();
         }
     }
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) > budget) {

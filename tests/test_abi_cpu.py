@@ -293,3 +293,38 @@ def test_c_example_compiles_and_links_against_the_abi(tmp_path):
     links libipt.so: the boundary is usable without Python or torch."""
     ipt.lib()
     _build_c_example(tmp_path)
+
+
+def test_edited_plans_rejected_before_device():
+    """validate_plan: each stage's variant must fit its shape -- stages 1 and 3
+    cycle following (identity only when a swapped dimension is 1), stage 2 tile / swap
+    (square tiles) / cycle following (identity only when m or n is 1).  Rejected before
+    any device use (IPT_ERR_INVALID_ARG = 1); a valid plan gets to the device query
+    (IPT_ERR_NO_DEVICE = 6 without a GPU)."""
+    L = ipt.lib()
+    null = ctypes.c_void_p(0)
+    p = ipt.plan(720, 1800, 4, -1, m=120, n=200)
+    assert [ipt.VARIANTS[v] for v in p.variant] == ["cycle_global", "tile_onchip", "cycle_global"]
+    ok = L.ipt_transpose_plan(ctypes.c_void_p(256), ctypes.byref(p), null, 0, null)
+    assert ok in (0, 6)
+    for st, v in [(0, 1), (2, 1), (0, 4), (0, 0), (2, 0), (1, 0), (1, 4), (1, 2), (0, 7), (1, -1)]:
+        bad = ipt.Plan.from_buffer_copy(p)
+        bad.variant[st] = v
+        assert L.ipt_transpose_plan(ctypes.c_void_p(256), ctypes.byref(bad), null, 0, null) == 1, (st, v)
+    sq = ipt.plan(720, 1800, 4, -1, m=120, n=120)
+    sq.variant[1] = 4                                   # square tiles may be swapped
+    assert L.ipt_transpose_plan(ctypes.c_void_p(256), ctypes.byref(sq), null, 0, null) in (0, 6)
+    one = ipt.plan(720, 1800, 4, -1, m=720, n=1800)     # stages 1 and 3 identities
+    assert [ipt.VARIANTS[v] for v in one.variant][0] == "identity"
+    assert L.ipt_transpose_plan(ctypes.c_void_p(256), ctypes.byref(one), null, 0, null) in (0, 6)
+
+
+def test_graph_wrapper_checks_sizes_without_gpu():
+    import torch
+
+    p = ipt.plan(36, 10, 4, -1)
+    t = torch.zeros(359, dtype=torch.int32)
+    with pytest.raises(ipt.IptError):
+        ipt.Graph(t, 36, 10, p)                         # 359 < 360 elements
+    with pytest.raises(ipt.IptError):
+        ipt.Graph(torch.zeros(360, dtype=torch.int32), 10, 36, p)   # plan for 36 x 10

@@ -426,14 +426,34 @@ def test_ipt_010_cluster_tiles(monkeypatch, split, eb, batch, A, B):
 # ---------------------------------------- unaligned super-elements (S % 16 != 0)
 @pytest.mark.parametrize("batch,A,B,s,eb", [(1, 61, 47, 131, 4), (3, 20, 30, 17, 4), (2, 9, 11, 4999, 4),
                                             (4, 33, 31, 65, 4), (1, 50, 70, 63, 8), (2, 40, 44, 1001, 8),
-                                            (1, 256, 131, 131, 4)])
-def test_ipt_100_unaligned_realigning_walker(batch, A, B, s, eb):
-    """4-byte-granular super-elements whose start phases differ mod 16 B use the
-    realigning warp walker (covering 16-B loads, shared-memory carry, partial stores)."""
+                                            (1, 256, 131, 131, 4), (1, 97, 103, 127, 4),
+                                            (2, 30, 41, 509, 4), (1, 23, 29, 1021, 4)])
+@pytest.mark.parametrize("seg", ["0", "2"])
+def test_ipt_100_unaligned_realigning_walker(monkeypatch, seg, batch, A, B, s, eb):
+    """4-byte-granular super-elements whose start phases differ mod 16 B: the realigning
+    flag walker (IPT_CYC_SEG=0: covering 16-B loads, shared-memory carry, partial stores)
+    and the segmented unaligned walker (2: covering loads, lane funnel shifts, edge words;
+    one chunk up to 508 words, 508-word chunks beyond)."""
+    monkeypatch.setenv("IPT_CYC_SEG", seg)
     a = gen(batch * A * B * s, eb)
     t = to_dev(a, eb)
     ipt.ipt_100_(t, batch, A, B, s)
     assert np.array_equal(to_np(t, eb), oracle.permute_inplace(a.copy(), batch, A, B, s))
+
+
+@pytest.mark.parametrize("seg", ["0", "2"])
+@pytest.mark.parametrize("off,batch,A,B,s", [(1, 1, 61, 47, 32), (3, 2, 30, 20, 64), (2, 1, 40, 31, 7)])
+def test_ipt_100_misaligned_base(monkeypatch, seg, off, batch, A, B, s):
+    """Data starting 4-12 bytes past a 16-byte boundary (16-byte multiple super-elements at
+    shifted phases): the unaligned walkers, bit-exact, neighbours untouched."""
+    monkeypatch.setenv("IPT_CYC_SEG", seg)
+    n = batch * A * B * s
+    a = gen(n + 8, 4)
+    t = to_dev(a, 4)
+    ipt.ipt_100_(t[off:off + n], batch, A, B, s)
+    got = to_np(t, 4)
+    assert np.array_equal(got[off:off + n], oracle.permute_inplace(a[off:off + n].copy(), batch, A, B, s))
+    assert np.array_equal(got[:off], a[:off]) and np.array_equal(got[off + n:], a[off + n:])
 
 
 @pytest.mark.parametrize("eb,batch,A,B", [(4, 2, 4999, 32), (4, 3, 1999, 31), (8, 2, 3001, 17),

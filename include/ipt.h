@@ -70,8 +70,12 @@ typedef enum {
 /* How one stage is executed. */
 typedef enum {
     IPT_VAR_IDENTITY = 0,      /* stage elided: a swapped dimension is 1 */
-    IPT_VAR_TILE_ONCHIP = 1,   /* whole tile staged in shared memory (BS, Fig. 1) */
-    IPT_VAR_CYCLE_ONCHIP = 2,  /* PTTWAC inside a tile, flag bits in shared memory */
+    IPT_VAR_TILE_ONCHIP = 1,   /* whole tile staged on chip (BS, Fig. 1): one CTA, a
+                                  cluster, a group of CTAs, or every SM with shared memory +
+                                  tensor memory (tiles up to ~70 MB) */
+    /* 2: reserved -- the paper's in-tile PTTWAC with flags in local memory (Sec. 5.1,
+       P:172-198) is not built on B200: every tile that fits an on-chip flag bitmap also
+       fits on chip itself; plans with variant 2 are rejected */
     IPT_VAR_CYCLE_GLOBAL = 3,  /* PTTWAC over super-elements, flag bits in global memory */
     IPT_VAR_SQUARE_SWAP = 4    /* square tiles (m == n, any size): symmetric swaps across the
                                   diagonal, cycles of length 2; with m = M = N = n the

@@ -27,7 +27,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libipt.so")
 
 IPT_OK = 0
-VARIANTS = {0: "identity", 1: "tile_onchip", 2: "cycle_onchip", 3: "cycle_global", 4: "square_swap"}
+VARIANTS = {0: "identity", 1: "tile_onchip", 3: "cycle_global", 4: "square_swap"}   # 2: reserved
 
 
 class IptError(RuntimeError):

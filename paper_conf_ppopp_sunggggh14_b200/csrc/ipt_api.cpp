@@ -1072,7 +1072,6 @@ int ipt__stage_kernel(const ipt_plan_t *plan, int64_t count, const void *d_base,
     switch (plan->variant[stage]) {
         case IPT_VAR_TILE_ONCHIP: name = tile_kernel_name(sd[stage], device); break;
         case IPT_VAR_SQUARE_SWAP: name = square_kernel_name(sd[stage]); break;
-        case IPT_VAR_CYCLE_ONCHIP:
         case IPT_VAR_CYCLE_GLOBAL: name = cycle_kernel_name(sd[stage], device); break;
         default: break;
     }

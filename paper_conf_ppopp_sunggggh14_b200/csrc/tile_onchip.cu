@@ -70,7 +70,9 @@ struct TileParams {
                           // to a second buffer after the data; 16 = timeline
                           // trace (results valid, see ipt__tile_trace)
     unsigned long long *trace;
-    uint32_t rows_a;      // tile_group_rf: slice rows staged in shared memory by TMA (rest: registers)
+    uint32_t rows_a;      // tile_group_rf: slice rows staged in shared memory by TMA (rest: TMEM)
+    uint32_t rows_b;      // tile_group_rf: rows per chunk of the TMEM part
+    uint32_t cpan;        // tile_group_rf: panels per chunk of the TMEM part
     uint32_t zero;        // 0 at run time, opaque to the compiler (load-completion dependency)
 };
 
@@ -713,6 +715,12 @@ __global__ void __launch_bounds__(512, 1) tile_group_tma(const TileParams p, con
 // is brought back (tcgen05.ld), stored into the freed shared memory in the same panel layout
 // and written out the same way.  Tiles of a group run one after another (a batch: the
 // spread of the CTAs overlaps one tile's stores with the next tile's loads across the GPU).
+__device__ __forceinline__ void tma_load_3d_t(uint32_t sdst, const CUtensorMap *tm, int32_t x, int32_t y,
+                                              int32_t z, uint32_t sbar) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];"
+        :: "r"(sdst), "l"(tm), "r"(x), "r"(y), "r"(z), "r"(sbar) : "memory");
+}
 __device__ __forceinline__ void tm_st4(uint32_t taddr, const uint4 &v) {
     asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1, %2, %3, %4};"
                  :: "r"(taddr), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
@@ -726,14 +734,39 @@ __device__ __forceinline__ uint4 tm_ld4(uint32_t taddr) {
 
 constexpr int kRfBatch = 8;   // part-B vectors per thread in registers at a time
 
-template <int EB, int RV>
+// Part B is handled in chunks (cb rows x cpan panels of the slice, staged through a
+// region of shared memory after part A's): chunk k's vectors are numbered consecutively
+// from base_k (E = base_k + row * ncols_k + col; every base a multiple of 512, so no
+// thread's TMEM column group is shared by two chunks -- tcgen05.st writes all 32 lanes),
+// thread E % 512 holds vector E in its TMEM columns 4 * (E / 512) .. +3.
+struct RfChunk {
+    uint32_t r0, nr, c0, nc, base;   // rows / vector columns of part B, first E
+};
+__device__ __forceinline__ RfChunk rf_chunk(const TileParams &p, uint32_t k, uint32_t rb, uint32_t cvec) {
+    const uint32_t cw = p.cpan * p.q;                              // chunk width (vectors)
+    const uint32_t npc = (cvec + cw - 1) / cw;                     // panel chunks per row chunk
+    RfChunk c{};
+    uint32_t base = 0;
+    for (uint32_t j = 0; j <= k; ++j) {
+        const uint32_t kr = j / npc, kc = j % npc;
+        c.r0 = kr * p.rows_b;
+        c.nr = min(p.rows_b, rb - c.r0);
+        c.c0 = kc * cw;
+        c.nc = min(cw, cvec - c.c0);
+        c.base = base;
+        base += (c.nr * c.nc + 511) / 512 * 512;
+    }
+    return c;
+}
+
+template <int EB, int RV, bool CH>
 __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, const __grid_constant__ CUtensorMap tmap) {
     constexpr int V = 16 / EB;
     static_assert(RV % kRfBatch == 0 && RV <= 32, "TMEM holds 32 vectors per thread");
     extern __shared__ __align__(128) unsigned char smem[];
     const uint32_t s0 = smem_u32(smem);
     const uint32_t K = p.K, rank = blockIdx.x % K, gid = blockIdx.x / K, ng = gridDim.x / K;
-    const uint32_t warp = threadIdx.x >> 5;
+    const uint32_t warp = threadIdx.x >> 5, tid = threadIdx.x;
     const uint32_t mv = p.m / V, nvr = p.n / V;
     uint32_t b0, b1, c0, c1;
     if (!p.colsplit) {
@@ -749,7 +782,10 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
     const uint32_t rows = (b1 - b0) * V, r0 = b0 * V;
     const uint32_t ra = min(p.rows_a, rows), rb = rows - ra;        // rows in smem / TMEM
     const uint32_t nvb = rb * cvec;                                    // part-B vectors of the slice
-    const uint32_t pstride_b = ((rb * q * 16) + 127) & ~127u;
+    // CH: part B in several chunks (compiled separately: the one-chunk kernel stays lean)
+    const uint32_t nchunk = !rb ? 0 : (!CH ? 1 : ((rb + p.rows_b - 1) / p.rows_b) *
+                                                 ((cvec + p.cpan * q - 1) / (p.cpan * q)));
+    const uint32_t pstride_b = (((CH ? p.rows_b : rb) * q * 16) + 127) & ~127u;
     const FastDiv32 divq = make_fastdiv32_dev(q), divc = make_fastdiv32_dev(cvec);
     const FastDiv32 diva = make_fastdiv32_dev(ra / V), divb = make_fastdiv32_dev(rb / V);
     __shared__ __align__(8) uint64_t mbar;
@@ -759,7 +795,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
                      :: "r"(smem_u32(&tmem_base)) : "memory");
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
     }
-    if (threadIdx.x == 0) {
+    if (tid == 0) {
         mbar_init(&mbar, 1);
         fence_mbar_init();
     }
@@ -771,27 +807,33 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
     uint32_t *ctr = p.gbar + gid * (kGroupCtrStride / 4);
     const uint32_t nt = gid < p.count ? (uint32_t)((p.count - gid + ng - 1) / ng) : 0;
     for (uint32_t i = 0; i < nt; ++i) {
-        char *g = tile_ptr(p, gid + (uint64_t)i * ng);
+        const uint64_t t = gid + (uint64_t)i * ng;
+        char *g = tile_ptr(p, t);
         // ---- part A: TMA boxes (rows_a rows of every panel; boxes may read past the slice)
-        if (threadIdx.x == 0) {
-            const uint64_t row0 = (uint64_t)(g - p.base) / ((uint64_t)p.n * EB) + r0;
+        if (tid == 0) {
             mbar_arrive_expect_tx(&mbar, p.npan * p.rows_a * q * 16);
             const uint32_t sbar = smem_u32(&mbar);
             for (uint32_t pn = 0; pn < p.npan; ++pn)
-                for (uint32_t r = 0; r < p.rows_a; r += p.box_rows)
-                    tma_load_2d(s0 + pn * p.pstride + r * q * 16, &tmap, (int32_t)((c0 + pn * q) * V),
-                                (int32_t)(row0 + r), sbar);
+                for (uint32_t r = 0; r < p.rows_a; r += p.box_rows) {
+                    const int32_t x = (int32_t)((c0 + pn * q) * V);
+                    const uint32_t dst = s0 + pn * p.pstride + r * q * 16;
+                    if (p.rres)   // strided batch: 3-D map (columns, rows, tiles)
+                        tma_load_3d_t(dst, &tmap, x, (int32_t)(r0 + r), (int32_t)t, sbar);
+                    else          // tiles stacked: 2-D map (columns, rows of all tiles)
+                        tma_load_2d(dst, &tmap, x, (int32_t)(t * p.m + r0 + r), sbar);
+                }
         }
-        // ---- part B: 16-byte loads, parked in TMEM batch by batch
-        const char *gb = g + ((size_t)(r0 + ra) * nvr + c0) * 16;
-        if (!(p.diag & 4)) {
+        // ---- part B: 16-byte loads parked in TMEM (thread E % 512 holds vector E in its
+        // columns 4 * (E / 512); with several chunks, chunk k's vectors start at base_k)
+        if (!(p.diag & 4) && !CH) {   // one chunk: every thread's vectors E < nvb
+            const char *gb = g + ((size_t)(r0 + ra) * nvr + c0) * 16;
 #pragma unroll 1
             for (int u0 = 0; u0 < RV; u0 += kRfBatch) {
                 if ((uint32_t)u0 * 512 >= nvb) break;
                 uint4 v[kRfBatch];
 #pragma unroll
                 for (int j = 0; j < kRfBatch; ++j) {
-                    const uint32_t e = threadIdx.x + (uint32_t)(u0 + j) * 512;
+                    const uint32_t e = tid + (uint32_t)(u0 + j) * 512;
                     v[j] = make_uint4(0, 0, 0, 0);
                     if (e < nvb) {
                         uint32_t r, c;
@@ -803,48 +845,103 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
                 for (int j = 0; j < kRfBatch; ++j) tm_st4(taddr + 4u * (uint32_t)(u0 + j), v[j]);
             }
             asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        } else if (!(p.diag & 4)) {
+            for (uint32_t k = 0; CH && k < nchunk; ++k) {
+                const RfChunk c = rf_chunk(p, k, rb, cvec);
+                const uint32_t n = c.nr * c.nc, uhi = (c.base + n + 511) / 512;
+                const FastDiv32 dnc = make_fastdiv32_dev(c.nc);
+                const char *gb = g + ((size_t)(r0 + ra + c.r0) * nvr + c0 + c.c0) * 16;
+#pragma unroll 1
+                for (uint32_t u0 = c.base / 512; u0 < uhi; u0 += kRfBatch) {
+                    uint4 v[kRfBatch];
+#pragma unroll
+                    for (int j = 0; j < kRfBatch; ++j) {
+                        const uint32_t E = tid + (u0 + j) * 512;
+                        v[j] = make_uint4(0, 0, 0, 0);
+                        if (E >= c.base && E < c.base + n) {
+                            uint32_t r, cc;
+                            fdivmod32(E - c.base, dnc, r, cc);
+                            v[j] = ld_cg<16>(gb + ((size_t)r * nvr + cc) * 16);
+                        }
+                    }
+#pragma unroll
+                    for (int j = 0; j < kRfBatch; ++j)
+                        if (u0 + j < uhi) tm_st4(taddr + 4u * (u0 + j), v[j]);   // warp-uniform bound
+                }
+            }
+            asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
         }
         mbar_wait(&mbar, i & 1);            // part A has landed
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         __syncthreads();
-        if (threadIdx.x == 0) {
+        if (tid == 0) {
             group_arrive(ctr, p.arrive_release != 0);
             if (!(p.diag & 1)) group_wait(ctr, K * (i + 1));   // all slices of the tile on chip
         }
         __syncthreads();
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        // ---- write-out: part A, then part B through the freed shared memory
+        // ---- write-out: part A, then part B (chunk by chunk) through the freed shared memory
         if (ra && !(p.diag & 2))
             write_out_pan<EB>(p, s0, g, q, divq, p.pstride, r0 / V, ra / V, diva, c0, cvec, NoProbe());
         __syncthreads();
+        if (!CH && nchunk) {   // one chunk: the whole part B through the freed shared memory
 #pragma unroll 1
-        for (int u0 = 0; u0 < RV; u0 += kRfBatch) {
-            if ((uint32_t)u0 * 512 >= nvb) break;
-            uint4 v[kRfBatch];
+            for (int u0 = 0; u0 < RV; u0 += kRfBatch) {
+                if ((uint32_t)u0 * 512 >= nvb) break;
+                uint4 v[kRfBatch];
 #pragma unroll
-            for (int j = 0; j < kRfBatch; ++j) v[j] = tm_ld4(taddr + 4u * (uint32_t)(u0 + j));
-            asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+                for (int j = 0; j < kRfBatch; ++j) v[j] = tm_ld4(taddr + 4u * (uint32_t)(u0 + j));
+                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 #pragma unroll
-            for (int j = 0; j < kRfBatch; ++j) {
-                const uint32_t e = threadIdx.x + (uint32_t)(u0 + j) * 512;
-                if (e < nvb) {
-                    uint32_t r, c, pn, pc;
-                    fdivmod32(e, divc, r, c);
-                    fdivmod32(c, divq, pn, pc);
-                    sts128(s0 + pn * pstride_b + (r * q + pc) * 16, v[j]);
+                for (int j = 0; j < kRfBatch; ++j) {
+                    const uint32_t e = tid + (uint32_t)(u0 + j) * 512;
+                    if (e < nvb) {
+                        uint32_t r, c, pn, pc;
+                        fdivmod32(e, divc, r, c);
+                        fdivmod32(c, divq, pn, pc);
+                        sts128(s0 + pn * pstride_b + (r * q + pc) * 16, v[j]);
+                    }
                 }
             }
+            __syncthreads();
+            if (!(p.diag & 2))
+                write_out_pan<EB>(p, s0, g, q, divq, pstride_b, (r0 + ra) / V, rb / V, divb, c0, cvec, NoProbe());
         }
-        __syncthreads();
-        if (rb && !(p.diag & 2))
-            write_out_pan<EB>(p, s0, g, q, divq, pstride_b, (r0 + ra) / V, rb / V, divb, c0, cvec, NoProbe());
+        for (uint32_t k = 0; CH && k < nchunk; ++k) {
+            const RfChunk c = rf_chunk(p, k, rb, cvec);
+            const uint32_t n = c.nr * c.nc, uhi = (c.base + n + 511) / 512;
+            const FastDiv32 dnc = make_fastdiv32_dev(c.nc);
+#pragma unroll 1
+            for (uint32_t u0 = c.base / 512; u0 < uhi; u0 += kRfBatch) {
+                uint4 v[kRfBatch];
+#pragma unroll
+                for (int j = 0; j < kRfBatch; ++j)
+                    if (u0 + j < uhi) v[j] = tm_ld4(taddr + 4u * (u0 + j));
+                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+                for (int j = 0; j < kRfBatch; ++j) {
+                    const uint32_t E = tid + (u0 + j) * 512;
+                    if (u0 + j < uhi && E >= c.base && E < c.base + n) {
+                        uint32_t r, cc, pn, pc;
+                        fdivmod32(E - c.base, dnc, r, cc);
+                        fdivmod32(cc, divq, pn, pc);
+                        sts128(s0 + pn * pstride_b + (r * q + pc) * 16, v[j]);
+                    }
+                }
+            }
+            __syncthreads();
+            if (!(p.diag & 2))
+                write_out_pan<EB>(p, s0, g, q, divq, pstride_b, (r0 + ra + c.r0) / V, c.nr / V,
+                                  make_fastdiv32_dev(c.nr / V), c0 + c.c0, c.nc, NoProbe());
+            __syncthreads();
+        }
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         __syncthreads();
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     }
     if (warp == 0)
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tmem_base) : "memory");
-    if (p.gexit && threadIdx.x == 0) {   // self-resetting counters (see group_loop)
+    if (p.gexit && tid == 0) {   // self-resetting counters (see group_loop)
         uint32_t *ex = p.gexit + gid * (kGroupCtrStride / 4);
         if (atomicAdd(ex, 1u) == K - 1) {
             atomicExch(ctr, 0u);
@@ -1800,12 +1897,16 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
 struct RfCfg {
     int K = 0, rv = 0;
     bool colsplit = false;
-    uint32_t q = 0, npan = 0, rows_a = 0, box_rows = 0;
+    uint32_t q = 0, npan = 0, rows_a = 0, rows_b = 0, cpan = 0, box_rows = 0;
     size_t pstride = 0, smem = 0;
 };
 constexpr int kRfThreads = 512;
 constexpr int kRfMaxRV = 32;   // part-B vectors per thread in TMEM (128 columns x 4 B)
 
+// Configuration of tile_group_rf: the largest part A in shared memory (TMA boxes of <= 256
+// rows, 128-byte aligned), part B in TMEM (at most 32 vectors per thread, every chunk
+// padded to 512 vectors) staged through part A's region after its write-out, in row (or
+// panel) chunks as large as shared memory allows.
 static RfCfg rf_search(int64_t A, int64_t B, int eb, int device, bool cs) {
     RfCfg c;
     const DevProps dp = dev_props(device);
@@ -1818,9 +1919,11 @@ static RfCfg rf_search(int64_t A, int64_t B, int eb, int device, bool cs) {
     const uint32_t npan = (uint32_t)((cvec + maxw - 1) / maxw);
     const uint32_t q = (uint32_t)(((cvec + npan - 1) / npan) | 1);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin) - 1024;
-    auto pst = [&](int64_t r) { return (size_t)((r * q * 16 + 127) & ~(int64_t)127); };
+    const int64_t maxchunks = 32;
+    auto pst = [&](int64_t r) { return (int64_t)((r * q * 16 + 127) & ~(int64_t)127); };
     for (int64_t ra = rows / V * V; ra >= V; ra -= V) {
-        if ((long)(npan * pst(ra)) > budget) continue;
+        const int64_t abytes = npan * pst(ra);
+        if (abytes > budget) continue;
         uint32_t br = 0;                                   // TMA box rows (128-B aligned boxes)
         if (ra <= 256) br = (uint32_t)ra;
         else
@@ -1828,17 +1931,42 @@ static RfCfg rf_search(int64_t A, int64_t B, int eb, int device, bool cs) {
                 if (ra % b == 0) { br = b; break; }
         if (!br) continue;
         const int64_t rb = rows - ra;
-        const int64_t rv = (rb * cvec + kRfThreads - 1) / kRfThreads;
-        if (rv > kRfMaxRV || (long)(npan * pst(rb)) > budget) return c;   // fewer rows in smem only adds registers
+        if ((rb * cvec + kRfThreads - 1) / kRfThreads > kRfMaxRV) return c;   // smaller A only adds TMEM
+        const int64_t room = budget;
+        const int64_t maxvec = INT64_MAX;   // vectors per chunk
+        int64_t cb = 0, cp = 0;
+        if (rb > 0) {
+            if (npan * pst(V) <= room && npan * V * cvec <= maxvec) {   // chunks of whole rows
+                cp = npan;
+                cb = V;
+                while (cb + V <= rb && npan * pst(cb + V) <= room && (cb + V) * cvec <= maxvec) cb += V;
+            } else if (pst(rb) <= room) {                                 // chunks of whole panels
+                cb = rb;
+                cp = std::max<int64_t>(1, std::min<int64_t>(room / pst(rb), maxvec / (rb * q)));
+                if (rb * q > maxvec) continue;
+            } else {
+                continue;
+            }
+            const int64_t cw = cp * q;
+            const int64_t nch = ((rb + cb - 1) / cb) * ((cvec + cw - 1) / cw);
+            if (nch > maxchunks) continue;
+            int64_t cols = 0;   // TMEM columns: every chunk padded to a multiple of 512 vectors
+            for (int64_t r = 0; r < rb; r += cb)
+                for (int64_t cc = 0; cc < cvec; cc += cw)
+                    cols += (std::min(cb, rb - r) * std::min(cw, cvec - cc) + kRfThreads - 1) / kRfThreads;
+            if (cols > kRfMaxRV) continue;
+        }
         c.K = K;
         c.colsplit = cs;
         c.q = q;
         c.npan = npan;
         c.rows_a = (uint32_t)ra;
+        c.rows_b = (uint32_t)std::max<int64_t>(cb, V);
+        c.cpan = (uint32_t)std::max<int64_t>(cp, 1);
         c.box_rows = br;
-        c.rv = (int)rv;
-        c.pstride = pst(ra);
-        c.smem = std::max(npan * pst(ra), npan * pst(rb));
+        c.rv = (int)((rb * cvec + kRfThreads - 1) / kRfThreads);
+        c.pstride = (size_t)pst(ra);
+        c.smem = (size_t)std::max<int64_t>(abytes, rb > 0 ? std::min<int64_t>(cp, npan) * pst(cb) : 0);
         return c;
     }
     return c;
@@ -1856,7 +1984,7 @@ static RfCfg rf_cfg(int64_t A, int64_t B, int eb, int device) {
     }
     const int K = dev_props(device).sms;
     const bool row_first = A * eb / K >= 64;   // as group_choose: row-split pieces >= 64 B
-    RfCfg c = rf_search(A, B, eb, device, !row_first);
+    RfCfg c = rf_search(A, B, eb, device, !row_first);   // the natural split direction first
     if (!c.K) c = rf_search(A, B, eb, device, row_first);
     std::lock_guard<std::mutex> lk(mu);
     cache[key] = c;
@@ -1867,25 +1995,42 @@ template <int EB>
 cudaError_t launch_group_rf(const StageDesc &d, TileParams p, const RfCfg &c, void *ws, cudaStream_t st,
                             int device) {
     if (!ws || !c.K) return cudaErrorInvalidValue;
-    if (d.outer > 1 && d.ostride != d.inner * (int64_t)p.tile_bytes) return cudaErrorNotSupported;
+    const bool packed = d.outer <= 1 || d.ostride == d.inner * (int64_t)p.tile_bytes;
+    if (!packed && d.inner != 1) return cudaErrorNotSupported;
     auto enc = tensor_map_encoder();
     if (!enc) return cudaErrorNotSupported;
     const int V = 16 / EB;
     CUtensorMap tm;
-    const uint64_t total_rows = (uint64_t)(d.outer * d.inner) * (uint64_t)d.A;
-    cuuint64_t dims[2] = {(cuuint64_t)d.B, (cuuint64_t)total_rows};
-    cuuint64_t strides[1] = {(cuuint64_t)(d.B * EB)};
-    cuuint32_t box[2] = {c.q * (uint32_t)V, c.box_rows};
-    cuuint32_t estr[2] = {1, 1};
-    CUresult r = enc(&tm, EB == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 2, d.base,
-                     dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    CUresult r;
+    if (packed) {   // tiles stacked: (columns, rows of all tiles)
+        const uint64_t total_rows = (uint64_t)(d.outer * d.inner) * (uint64_t)d.A;
+        cuuint64_t dims[2] = {(cuuint64_t)d.B, (cuuint64_t)total_rows};
+        cuuint64_t strides[1] = {(cuuint64_t)(d.B * EB)};
+        cuuint32_t box[2] = {c.q * (uint32_t)V, c.box_rows};
+        cuuint32_t estr[2] = {1, 1};
+        r = enc(&tm, EB == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 2, d.base,
+                dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        p.rres = 0;
+    } else {        // strided batch of single tiles: (columns, rows, tiles), tile stride ostride
+        if (d.ostride % 16) return cudaErrorNotSupported;
+        cuuint64_t dims[3] = {(cuuint64_t)d.B, (cuuint64_t)d.A, (cuuint64_t)d.outer};
+        cuuint64_t strides[2] = {(cuuint64_t)(d.B * EB), (cuuint64_t)d.ostride};
+        cuuint32_t box[3] = {c.q * (uint32_t)V, c.box_rows, 1};
+        cuuint32_t estr[3] = {1, 1, 1};
+        r = enc(&tm, EB == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 3, d.base,
+                dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        p.rres = 1;
+    }
     if (r != CUDA_SUCCESS) return cudaErrorNotSupported;
     p.q = c.q;
     p.npan = c.npan;
     p.pstride = (uint32_t)c.pstride;
     p.box_rows = c.box_rows;
     p.rows_a = c.rows_a;
+    p.rows_b = c.rows_b;
+    p.cpan = c.cpan;
     p.colsplit = c.colsplit ? 1 : 0;
     p.K = (uint32_t)c.K;
     p.nbuf = 1;
@@ -1905,8 +2050,10 @@ cudaError_t launch_group_rf(const StageDesc &d, TileParams p, const RfCfg &c, vo
         if (e != cudaSuccess) return e;
     }
     const void *kern = nullptr;
-    const int rv = (c.rv + kRfBatch - 1) / kRfBatch * kRfBatch;
-#define IPT_RF(R) if (rv == R) kern = (const void *)tile_group_rf<EB, R>;
+    const int rv = std::max(kRfBatch, (c.rv + kRfBatch - 1) / kRfBatch * kRfBatch);
+    const int64_t rbm = (int64_t)(c.colsplit ? d.A : ((d.A / V + c.K - 1) / c.K) * V) - c.rows_a;   // max rows in TMEM
+    const bool ch = rbm > (int64_t)c.rows_b || c.cpan < c.npan;
+#define IPT_RF(R) if (rv == R) kern = ch ? (const void *)tile_group_rf<EB, R, true> : (const void *)tile_group_rf<EB, R, false>;
     IPT_RF(8) IPT_RF(16) IPT_RF(24) IPT_RF(32)
 #undef IPT_RF
     if (!kern) return cudaErrorNotSupported;
@@ -1933,8 +2080,8 @@ cudaError_t launch_group_rf(const StageDesc &d, TileParams p, const RfCfg &c, vo
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     if (env_int("IPT_DEBUG", 0))
-        fprintf(stderr, "[ipt] tile_group_rf m=%u n=%u K=%d colsplit=%d q=%u npan=%u rows_a=%u box=%u rv=%d smem=%zu tiles=%llu\n",
-                p.m, p.n, c.K, p.colsplit, c.q, c.npan, c.rows_a, c.box_rows, rv, c.smem,
+        fprintf(stderr, "[ipt] tile_group_rf m=%u n=%u K=%d colsplit=%d q=%u npan=%u rows_a=%u chunk=%ux%u box=%u rv=%d smem=%zu tiles=%llu\n",
+                p.m, p.n, c.K, p.colsplit, c.q, c.npan, c.rows_a, c.rows_b, c.cpan, c.box_rows, rv, c.smem,
                 (unsigned long long)p.count);
     void *args[] = {&p, &tm};
     p.diag = (int)env_int("IPT_TILE_DIAG", 0);
@@ -2054,6 +2201,7 @@ int tile_group_k(int64_t A, int64_t B, int eb, uint64_t count, int device, int *
 int tile_onchip_path(int64_t A, int64_t B, int eb, int device) {
     DevProps dp = dev_props(device);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
+    if (env_int("IPT_TILE_RF_FORCE", 0) && tile_rf_fits(A, B, eb, device)) return 7;   // tests
     if (vec_ok(A, B, eb) && (long)fast_smem(A, B, eb) <= budget) return 2;
     if (tile_group_split(A, B, eb, device)) return 5;
     if (tile_cluster_k(A, B, eb, device)) return 3;
@@ -2074,6 +2222,8 @@ bool tile_rf_fits(int64_t A, int64_t B, int eb, int device) { return rf_cfg(A, B
 const char *tile_kernel_name(const StageDesc &d, int device) {
     const DevProps dp = dev_props(device);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
+    if (env_int("IPT_TILE_RF_FORCE", 0) && fast_ok(d) && (d.eb == 4 || d.eb == 8) && rf_cfg(d.A, d.B, d.eb, device).K)
+        return "tile_group_rf";
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) <= budget) {
         const size_t smem = fast_smem(d.A, d.B, d.eb);
         if (smem > 113 * 1024 && env_int("IPT_TILE_STREAM", 1) && tile_mode() != MODE_TMA)
@@ -2098,8 +2248,8 @@ const char *tile_kernel_name(const StageDesc &d, int device) {
     }
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) > budget && tile_cluster_k(d.A, d.B, d.eb, device))
         return "tile_onchip_cluster";
-    if (fast_ok(d) && (d.eb == 4 || d.eb == 8) && (long)generic_smem(d.A, d.B, d.eb) > budget && packed &&
-        rf_cfg(d.A, d.B, d.eb, device).K)
+    if (fast_ok(d) && (d.eb == 4 || d.eb == 8) && (long)generic_smem(d.A, d.B, d.eb) > budget &&
+        (packed || d.inner == 1) && rf_cfg(d.A, d.B, d.eb, device).K)
         return "tile_group_rf";
     if ((long)generic_smem(d.A, d.B, d.eb) > budget) return "tile_generic_cluster";
     return "tile_onchip_generic";
@@ -2132,6 +2282,11 @@ cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, in
     }
     p.arrive_release = (int)env_int("IPT_TILE_ARRIVE_RELEASE", 0);
     const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
+    if (env_int("IPT_TILE_RF_FORCE", 0) && fast_ok(d) && (d.eb == 4 || d.eb == 8)) {   // tests
+        const RfCfg c = rf_cfg(d.A, d.B, d.eb, device);
+        if (c.K) return d.eb == 4 ? launch_group_rf<4>(d, p, c, ws, st, device)
+                                  : launch_group_rf<8>(d, p, c, ws, st, device);
+    }
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) <= budget) {
         const int V = 16 / d.eb;
         p.q = fast_q(d.B, d.eb);

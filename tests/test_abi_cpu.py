@@ -171,9 +171,13 @@ def test_plan_prefers_vector_tiles_on_large_f32():
 
 
 def test_workspace_batch_scales():
-    p = ipt.plan(4096, 3000, 4)
+    # flag bits scale with the batch (one per unit and matrix) ...
+    p = ipt.plan(4096, 3000, 4, m=256, n=3000)          # tile stage + cycle stage
     w1, w8 = ipt.workspace_bytes(p, 1), ipt.workspace_bytes(p, 8)
     assert w8 > w1 and w8 <= 8 * w1 + 256
+    # ... a one-stage whole-matrix plan (the tile on chip) needs only the group counters
+    p = ipt.plan(4096, 3000, 4)
+    assert p.n_stages == 1 and ipt.workspace_bytes(p, 512) == ipt.workspace_bytes(p, 1) == 8192
 
 
 def test_group_split_extends_on_chip_tiles():
@@ -192,7 +196,10 @@ def test_group_split_extends_on_chip_tiles():
     # up to ~148 x 227 KB with ONE slice buffer per CTA (single-buffered groups)
     p = ipt.plan(4096, 8192, 4, m=4096, n=2048)         # 32 MB: single-buffered group
     assert V[p.variant[1]] == "tile_onchip"
-    p = ipt.plan(8192, 8192, 4, m=8192, n=2048)         # 64 MB: beyond aggregate smem
+    # up to ~148 x (227 KB smem + 256 KB TMEM) for whole-GPU tiles (tile_group_rf)
+    p = ipt.plan(8192, 8192, 4, m=8192, n=2048)         # 64 MB: smem + tensor memory
+    assert V[p.variant[1]] == "tile_onchip" and ipt.stage_kernels(p)[1] == "tile_group_rf"
+    p = ipt.plan(8192, 8192, 4, m=8192, n=4096)         # 128 MB: beyond on-chip storage
     assert V[p.variant[1]] == "cycle_global"
     assert ipt.lib().ipt_stage_workspace_bytes(3, 120, 7200, 1, 4) >= 8192
     assert ipt.lib().ipt_stage_workspace_bytes(1, 4, 4, 5, 4) < 8192   # cycle stage: flags only

@@ -215,3 +215,45 @@ def test_edited_plan_rejected():
         with pytest.raises(ipt.IptError):
             ipt.transpose_(t, M, N, plan_=bad)
     assert _is_input(t, M, N, 4)                         # nothing was launched
+
+
+# ------------------------- whole-GPU tiles in shared memory + tensor memory (tile_group_rf)
+RF_CASES = [  # (M, N, eb, count, stride pad in elements, smem budget override or 0)
+    (4096, 3000, 4, 3, 0, 0),          # C5 matrices: row split, 16 rows by TMA + 12 in TMEM
+    (3000, 4096, 4, 2, 64, 0),         # strided batch: 3-D tensor map
+    (1800, 7200, 4, 1, 0, 0),          # C1: column split
+    (7200, 1800, 4, 1, 0, 0),
+    (1024, 16384, 4, 1, 0, 0),         # 67 MB: TMEM part written out in row chunks
+    (2048, 4096, 8, 1, 0, 0),          # float64
+    (720, 1800, 4, 5, 0, 20000),       # small tiles forced through the rf path with a small
+    (1200, 760, 8, 3, 8, 12000),       # smem budget: TMEM part in several row chunks
+    (720, 1800, 4, 2, 0, 60000),       # everything in shared memory (no TMEM part)
+]
+
+
+@pytest.mark.parametrize("M,N,eb,count,pad,smem", RF_CASES,
+                         ids=[f"{c[0]}x{c[1]}x{c[2]}b{c[3]}p{c[4]}s{c[5]}" for c in RF_CASES])
+def test_tile_group_rf(monkeypatch, M, N, eb, count, pad, smem):
+    """The whole tile of a 1-stage plan (m = M, n = N) held over every SM in shared memory
+    (TMA part) and TMEM (tcgen05.st / tcgen05.ld part): every element checked by the
+    definition, strided gaps untouched, then transposed back."""
+    monkeypatch.setenv("IPT_TILE_RF_FORCE", "1")
+    if smem:
+        monkeypatch.setenv("IPT_TILE_SMEM_MAX", str(smem))
+    dt = torch.int32 if eb == 4 else torch.int64
+    stride = M * N + pad
+    t = torch.empty(count * stride, dtype=dt, device="cuda")
+    for k in range(count):
+        seeded.fill_device_(t[k * stride:k * stride + M * N], M, N, eb, t0=k)
+    gaps = [t[k * stride + M * N:(k + 1) * stride].clone() for k in range(count)]
+    p = ipt.plan(M, N, eb, 0, m=M, n=N)
+    q = ipt.plan(N, M, eb, 0, m=N, n=M)
+    assert ipt.stage_kernels(p, count, t)[1] == "tile_group_rf"
+    ipt.transpose_batched_(t, count, M, N, stride_elems=stride, plan_=p)
+    torch.cuda.synchronize()
+    for k in range(count):
+        assert _definition(t[k * stride:k * stride + M * N], M, N, eb, k), k
+        assert torch.equal(t[k * stride + M * N:(k + 1) * stride], gaps[k])
+    ipt.transpose_batched_(t, count, N, M, stride_elems=stride, plan_=q)
+    for k in range(count):
+        assert _is_input(t[k * stride:k * stride + M * N], M, N, eb, t0=k), k

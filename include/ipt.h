@@ -210,17 +210,18 @@ ipt_status ipt_transpose_host_pipeline(void *const *h_ptrs, const int64_t *Ms, c
  * Replaying it (ipt_graph_launch) transposes those matrices in place with one
  * cudaGraphLaunch -- no per-call planning, validation or kernel-launch overhead.  The graph
  * is bound to the pointers.  Workspace: the caller's d_workspace (>= ipt_workspace_bytes;
- * then replays must not overlap each other or other calls using it), or NULL = a
- * graph-owned allocation made and released inside every replay (memory allocation nodes),
- * so replays on any stream never share flags or counters with other work.  Captured
+ * then replays must not overlap each other or other calls using it), or NULL = a buffer
+ * owned by the graph (allocated here, freed by ipt_graph_destroy), so replays never share
+ * flags or counters with direct calls or other graphs (replays of ONE graph must be
+ * stream-ordered with each other).  A libipt call captured by the caller (e.g.
+ * torch.cuda.graph) with a NULL workspace instead allocates and frees its flags inside the
+ * captured sequence (memory allocation nodes; costlier per replay).  Captured
  * launches never use the library's per-stream self-resetting counters (they zero their
  * counters with memset nodes).  Segment lists of segmented cycle stages are used only if a
  * direct call built them already (else the flag kernel is captured): run the plan once
  * before capturing to get identical kernels.  ipt_graph_destroy frees everything the
  * handle owns (the caller synchronises first).  Note that an M x N graph replayed twice
- * applies the M x N transposition twice; pair it with an N x M graph.
- * The same rules apply to any libipt call captured by the caller (e.g. torch.cuda.graph):
- * with a NULL workspace the captured sequence allocates and frees its own flags. */
+ * applies the M x N transposition twice; pair it with an N x M graph. */
 ipt_status ipt_graph_create(void *d_base, int64_t count, int64_t stride_bytes, const ipt_plan_t *plan,
                             void *d_workspace, size_t ws_bytes, void **out);
 ipt_status ipt_graph_launch(void *graph, void *stream);

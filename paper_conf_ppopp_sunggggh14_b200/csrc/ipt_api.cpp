@@ -984,6 +984,7 @@ ipt_status ipt_asta_to_soa(void *d_ptr, int64_t M, int64_t N, int64_t m, int ele
 // capturing to get the same kernels as the uncaptured call.
 struct GraphHandle {
     cudaGraphExec_t exec;
+    void *ws;   // workspace owned by the graph (freed by ipt_graph_destroy), or nullptr
 };
 
 ipt_status ipt_graph_create(void *d_base, int64_t count, int64_t stride_bytes, const ipt_plan_t *plan,
@@ -999,12 +1000,28 @@ ipt_status ipt_graph_create(void *d_base, int64_t count, int64_t stride_bytes, c
     if (count > 1 && (stride_bytes < mat || stride_bytes % plan->elem_bytes)) return IPT_ERR_INVALID_ARG;
     const int device = current_device();
     if (device < 0) return IPT_ERR_NO_DEVICE;
-    if (d_workspace && ws_bytes < batched_ws(plan, count)) return IPT_ERR_NO_MEMORY;
+    const size_t need = batched_ws(plan, count);
+    if (d_workspace && ws_bytes < need) return IPT_ERR_NO_MEMORY;
+    // without a caller workspace the graph owns one (allocated here, outside the capture,
+    // freed by ipt_graph_destroy): replays of this graph are ordered on the caller's stream
+    // and never share it with direct calls or other graphs (allocation nodes inside the
+    // graph -- what run_plan does for a caller's capture -- cost 0.2-1.4 ms per replay)
+    void *own = nullptr;
+    if (!d_workspace && need) {
+        if (cudaMalloc(&own, need) != cudaSuccess) {
+            cudaGetLastError();
+            return IPT_ERR_NO_MEMORY;
+        }
+        d_workspace = own;
+        ws_bytes = need;
+    }
     cudaStream_t cs;
     cudaError_t e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
-    if (e != cudaSuccess) return cuda_status(e);
-    // without a caller workspace, run_plan gives the graph its own workspace (allocation
-    // nodes); library-owned per-stream counters are never used under capture
+    if (e != cudaSuccess) {
+        if (own) cudaFree(own);
+        return cuda_status(e);
+    }
+    // library-owned per-stream counters are never used under capture (memset nodes instead)
     cudaGraph_t g = nullptr;
     e = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal);
     if (e == cudaSuccess) {
@@ -1015,11 +1032,13 @@ ipt_status ipt_graph_create(void *d_base, int64_t count, int64_t stride_bytes, c
     GraphHandle *h = nullptr;
     if (!s && e == cudaSuccess) {
         h = new GraphHandle{};
+        h->ws = own;
         e = cudaGraphInstantiate(&h->exec, g, 0);
         if (e != cudaSuccess) { delete h; h = nullptr; }
     }
     if (g) cudaGraphDestroy(g);
     cudaStreamDestroy(cs);   // nothing was launched on it: captured work lives in the graph
+    if ((s || e != cudaSuccess) && own) cudaFree(own);
     if (s) return s;
     if (e != cudaSuccess) return cuda_status(e);
     *out = h;
@@ -1035,6 +1054,10 @@ ipt_status ipt_graph_destroy(void *graph) {
     if (!graph) return IPT_OK;
     GraphHandle *h = (GraphHandle *)graph;
     cudaError_t e = cudaGraphExecDestroy(h->exec);
+    if (h->ws) {   // the caller synchronised: no replay still uses it
+        const cudaError_t f = cudaFree(h->ws);
+        if (e == cudaSuccess) e = f;
+    }
     delete h;
     return cuda_status(e);
 }

@@ -109,3 +109,17 @@ def test_bench_gpus_flag_spawns_ranks():
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2"],
                        capture_output=True, text=True, timeout=120, env=env, cwd=ROOT)
     assert r.returncode == 2
+
+
+def test_workloads_lists():
+    """The benched shape lists (inputs/workloads.py): the full SURVEY C2 classes, seeded
+    random pairs reproducible, in range, no duplicates; C5 = 512 x 4096 x 3000."""
+    from inputs import workloads as W
+
+    assert W.C5_SHAPE == (4096, 3000) and W.C5_COUNT == 512
+    assert W.sweep_random_pairs() == W.SWEEP_RANDOM and len(W.SWEEP_RANDOM) == 16
+    assert all(1000 <= a <= 20000 and 1000 <= b <= 20000 for a, b in W.SWEEP_RANDOM)
+    for s in W.TABLE2 + W.SWEEP_POW2 + W.SWEEP_FEW_FACTORS + W.SWEEP_LARGE + W.SWEEP_RANDOM:
+        assert s in W.SWEEP_ALL
+    assert len(set(W.SWEEP_ALL)) == len(W.SWEEP_ALL)
+    assert (9797, 13081) in W.SWEEP_ALL and (10007, 19997) in W.PRIMES

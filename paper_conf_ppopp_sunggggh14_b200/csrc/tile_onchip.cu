@@ -806,9 +806,19 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
     const uint32_t taddr = tmem_base + ((32u * (warp & 3)) << 16) + (warp >> 2) * 128u;
     uint32_t *ctr = p.gbar + gid * (kGroupCtrStride / 4);
     const uint32_t nt = gid < p.count ? (uint32_t)((p.count - gid + ng - 1) / ng) : 0;
+    // timeline trace (IPT_TILE_DIAG=16; tools/rf_trace.py): per CTA and tile, globaltimer at
+    // start, part B parked, part A landed, group complete, A written, B staged, B written
+    unsigned long long *tr = (p.diag & 16) && tid == 0 ? p.trace + (uint64_t)blockIdx.x * 256 : nullptr;
+    auto mark = [&](uint32_t i, int k) { if (tr && i < 31) tr[i * 8 + k] = global_ns(); };
+    if (tr) {   // last slot: the SM this CTA runs on
+        uint32_t smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        tr[31 * 8] = smid;
+    }
     for (uint32_t i = 0; i < nt; ++i) {
         const uint64_t t = gid + (uint64_t)i * ng;
         char *g = tile_ptr(p, t);
+        mark(i, 0);
         // ---- part A: TMA boxes (rows_a rows of every panel; boxes may read past the slice)
         if (tid == 0) {
             mbar_arrive_expect_tx(&mbar, p.npan * p.rows_a * q * 16);
@@ -848,6 +858,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
                 for (int j = 0; j < kRfBatch; ++j) tm_st4(taddr + 4u * (uint32_t)(u0 + j), v[j]);
             }
             asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+            mark(i, 1);
         } else if (!(p.diag & 4)) {
             for (uint32_t k = 0; CH && k < nchunk; ++k) {
                 const RfChunk c = rf_chunk(p, k, rb, cvec);
@@ -875,18 +886,21 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
             asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
         }
         mbar_wait(&mbar, i & 1);            // part A has landed
+        mark(i, 2);
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         __syncthreads();
         if (tid == 0) {
             group_arrive(ctr, p.arrive_release != 0);
             if (!(p.diag & 1)) group_wait(ctr, K * (i + 1));   // all slices of the tile on chip
         }
+        mark(i, 3);
         __syncthreads();
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         // ---- write-out: part A, then part B (chunk by chunk) through the freed shared memory
         if (ra && !(p.diag & 2))
             write_out_pan<EB>(p, s0, g, q, divq, p.pstride, r0 / V, ra / V, diva, c0, cvec, NoProbe());
         __syncthreads();
+        mark(i, 4);
         if (!CH && nchunk) {   // one chunk: the whole part B through the freed shared memory
 #pragma unroll 1
             for (int u0 = 0; u0 < RV; u0 += kRfBatch) {
@@ -907,6 +921,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
                 }
             }
             __syncthreads();
+            mark(i, 5);
             if (!(p.diag & 2))
                 write_out_pan<EB>(p, s0, g, q, divq, pstride_b, (r0 + ra) / V, rb / V, divb, c0, cvec, NoProbe());
         }
@@ -941,6 +956,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         __syncthreads();
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        mark(i, 6);
     }
     if (warp == 0)
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tmem_base) : "memory");

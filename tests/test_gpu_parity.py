@@ -795,15 +795,18 @@ SQ_SIDES = [2, 3, 7, 15, 16, 17, 63, 64, 65, 100, 127, 128, 129, 255, 256, 257, 
 
 
 @pytest.mark.parametrize("eb", [1, 2, 4, 8, 16])
-@pytest.mark.parametrize("path", ["auto", "tma", "vec", "elem", "tb512", "tb512nt512", "swz", "swz512", "noswz"])
+@pytest.mark.parametrize("path", ["auto", "tma", "vec", "elem", "elem_pf32", "elem_pf64", "elem_plain", "tb512",
+                                  "tb512nt512", "swz", "swz512", "noswz"])
 def test_square_swap_sides(monkeypatch, eb, path):
     """ipt_010 on square items through the swap kernel (TMA ring by default, register
     staged, element path): every side spans ragged block edges (g not a multiple of the
     block) and, for g % (16/b) != 0, the element path; batches fold several items into
     one launch (rows of a ragged last block belong to the next item)."""
     monkeypatch.setenv("IPT_SQ_FORCE", "1")
-    if path == "elem":
+    if path.startswith("elem"):
         monkeypatch.setenv("IPT_SQ_ELEM", "1")
+    if path.startswith("elem_p"):   # the element path's prefetching variants / the plain kernel
+        monkeypatch.setenv("IPT_SQ_ELEM_PF", {"elem_pf32": "32", "elem_pf64": "64", "elem_plain": "0"}[path])
     if path.startswith("tb512"):
         monkeypatch.setenv("IPT_SQ_TB", "512")
     if path == "tb512nt512":

@@ -7,7 +7,7 @@ if os.environ.get("_CHILD"):
     import torch
     import paper_conf_ppopp_sunggggh14_b200 as ipt
     TOT_BYTES = 800 << 20
-    dt = {4: torch.int32, 8: torch.int64, 16: torch.int64}
+    dt = {2: torch.int16, 4: torch.int32, 8: torch.int64, 16: torch.int64}
     res = {}
     for (g, eb) in ast.literal_eval(os.environ["SHAPES"]):
         cnt = max(1, TOT_BYTES // (g * g * eb))

@@ -40,7 +40,8 @@ def sweep_random_pairs(n: int = 16, seed: int = 1):
 SWEEP_RANDOM = sweep_random_pairs()
 
 # prime / prime-containing dims: correctness only ("degrade")
-PRIMES = [(19997, 1024), (1021, 4093), (1009, 7001), (10007, 19997)]
+PRIMES = [(19997, 1024), (1021, 4093), (1009, 7001), (10007, 19997),
+          (10007, 10007)]    # a prime-sided square: the swap kernel's element path
 
 
 def dedup(shapes):

@@ -27,7 +27,7 @@ from oracle import oracle  # noqa: E402
 
 AUTOTUNE = 8   # bench.py --autotune default
 
-SHAPES = ([(M, N, 4) for (M, N) in W.C1 + W.C3 + W.SWEEP_ALL + W.PRIMES + [(10007, 10007)]]
+SHAPES = ([(M, N, 4) for (M, N) in W.C1 + W.C3 + W.SWEEP_ALL + W.PRIMES]
           + [(M, N, 8) for (M, N) in W.C4])
 
 

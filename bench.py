@@ -320,7 +320,7 @@ def _stage_rec(ipt, p, cnt, t, a, b, eb, ms):
     return out
 
 
-def measure_matrix(ipt, torch, dev, M, N, eb, steps, warmup, autotune, l2_bytes, flush):
+def measure_matrix(ipt, torch, dev, M, N, eb, steps, warmup, autotune, l2_bytes, flush, graphs=False):
     """One matrix on its own: plans (measured), warm-up, `steps` transposes timed one by one
     with CUDA events (orientation alternating; cold L2 for L2-resident matrices), then two
     steps with per-stage events (both orientations), then a sampled definition check."""
@@ -370,6 +370,25 @@ def measure_matrix(ipt, torch, dev, M, N, eb, steps, warmup, autotune, l2_bytes,
         torch.cuda.synchronize()
         ms = [evs[i].elapsed_time(evs[i + 1]) for i in range(3)]
         stages[f"{a}x{b}"] = _stage_rec(ipt, plans[(a, b)], 1, t, a, b, eb, ms)
+    # the same steps replayed as captured CUDA graphs (ipt_graph_create / ipt_graph_launch:
+    # no host-side planning or launch API calls per transposition)
+    graph_ms = None
+    if graphs:
+        gr = {(a, b): ipt.Graph(t, a, b, plans[(a, b)]) for (a, b) in ((M, N), (N, M))}
+        gtot = 0.0
+        for s in range(steps):
+            a, b = (N, M) if orient else (M, N)
+            if resident:
+                flush.sum()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            gr[(a, b)].launch()
+            e1.record()
+            torch.cuda.synchronize()
+            gtot += e0.elapsed_time(e1)
+            orient = not orient
+        graph_ms = gtot
+        del gr
     ok = _verify(t, M, N, eb, orient)
     del t
     torch.cuda.empty_cache()
@@ -383,6 +402,8 @@ def measure_matrix(ipt, torch, dev, M, N, eb, steps, warmup, autotune, l2_bytes,
     }
     sbytes = sum(2 * M * N * eb * plans[(N, M) if (s % 2) else (M, N)].n_stages for s in range(steps))
     rec["hbm_frac_stage_scaled"] = round(sbytes / (tot / 1e3) / 1e9 / load_peaks()[0], 4)
+    if graph_ms:
+        rec["graph_eff_gbs"] = round(2 * M * N * eb * steps / (graph_ms / 1e3) / 1e9, 1)
     return rec, tot, 2 * M * N * eb * steps
 
 
@@ -395,8 +416,13 @@ def run_sub(ipt, torch, dev, name, steps, warmup, autotune):
     per, agg = {}, {"all": [0.0, 0], "squares": [0.0, 0], "rectangles": [0.0, 0]}
     ok = True
     t0 = time.perf_counter()
+    graphs = name in ("c1", "table2")   # single L2-sized matrices: also timed as CUDA graphs
+    gagg = [0.0, 0]
     for (M, N) in wl["shapes"]:
-        rec, ms, by = measure_matrix(ipt, torch, dev, M, N, eb, steps, warmup, autotune, l2, flush)
+        rec, ms, by = measure_matrix(ipt, torch, dev, M, N, eb, steps, warmup, autotune, l2, flush, graphs)
+        if "graph_eff_gbs" in rec:
+            gagg[0] += by / (rec["graph_eff_gbs"] * 1e9) * 1e3
+            gagg[1] += by
         per[f"{M}x{N}"] = rec
         ok &= rec["verified"]
         for k in ("all", "squares" if M == N else "rectangles"):
@@ -412,6 +438,9 @@ def run_sub(ipt, torch, dev, name, steps, warmup, autotune):
         for k in ("squares", "rectangles"):
             if agg[k][1]:
                 out[k] = round(agg[k][1] / (agg[k][0] / 1e3) / 1e9, 1)
+    if gagg[1]:
+        out["graph_value"] = round(gagg[1] / (gagg[0] / 1e3) / 1e9, 1)
+        out["graph_note"] = "the same steps replayed as captured CUDA graphs (ipt_graph_launch)"
     if name == "primes":
         out["note"] = "correctness-only class (P:319: prime dimensions degrade; SURVEY C14)"
     out["per_shape"] = per

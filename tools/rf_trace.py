@@ -64,3 +64,9 @@ if nt > 2:
     print(f"median load {np.median(load):.1f} writeA {np.median(wa):.1f} stageB {np.median(sb):.1f} writeB {np.median(wb):.1f}")
     rows = np.array([((c + 1) * (M // 4) // 148 - c * (M // 4) // 148) for c in range(148)])
     print("rows(V-blocks) of the slowest:", rows[order[-8:]], " fastest:", rows[order[:4]])
+if nt > 2 and os.environ.get("RF_TRACE_ALL"):
+    wt = wa + sb + wb
+    print("per SM (sm: write us):")
+    by = sorted(zip(smid, wt, load))
+    print(" ".join(f"{int(s)}:{w:.1f}" for s, w, _ in by))
+    np.save("gpurun_out/rf_sm_write.npy", np.array([[s, w, l] for s, w, l in by]))

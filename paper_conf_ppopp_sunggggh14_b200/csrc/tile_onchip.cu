@@ -769,9 +769,10 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
     const uint32_t warp = threadIdx.x >> 5, tid = threadIdx.x;
     const uint32_t mv = p.m / V, nvr = p.n / V;
     uint32_t b0, b1, c0, c1;
-    if (!p.colsplit) {
-        b0 = (uint32_t)((uint64_t)rank * mv / K);
-        b1 = (uint32_t)((uint64_t)(rank + 1) * mv / K);
+    if (!p.colsplit) {   // row slices in units of ralign V-row blocks (sector-aligned pieces)
+        const uint32_t ra_ = p.ralign ? p.ralign : 1u, units = mv / ra_;
+        b0 = (uint32_t)((uint64_t)rank * units / K) * ra_;
+        b1 = rank + 1 == K ? mv : (uint32_t)((uint64_t)(rank + 1) * units / K) * ra_;
         c0 = 0; c1 = nvr;
     } else {
         b0 = 0; b1 = mv;
@@ -1916,7 +1917,7 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
 struct RfCfg {
     int K = 0, rv = 0;
     bool colsplit = false;
-    uint32_t q = 0, npan = 0, rows_a = 0, rows_b = 0, cpan = 0, box_rows = 0;
+    uint32_t q = 0, npan = 0, rows_a = 0, rows_b = 0, cpan = 0, box_rows = 0, ralign = 0;
     size_t pstride = 0, smem = 0;
 };
 constexpr int kRfThreads = 512;
@@ -1926,13 +1927,15 @@ constexpr int kRfMaxRV = 32;   // part-B vectors per thread in TMEM (128 columns
 // rows, 128-byte aligned), part B in TMEM (at most 32 vectors per thread, every chunk
 // padded to 512 vectors) staged through part A's region after its write-out, in row (or
 // panel) chunks as large as shared memory allows.
-static RfCfg rf_search(int64_t A, int64_t B, int eb, int device, bool cs, bool chunks) {
+static RfCfg rf_search(int64_t A, int64_t B, int eb, int device, bool cs, bool chunks, int64_t ral) {
     RfCfg c;
     const DevProps dp = dev_props(device);
     const int K = dp.sms, V = 16 / eb;
     const int64_t mv = A / V, nvr = B / V;
+    if (!cs && (mv % ral || mv / ral < K)) return c;
     if ((cs ? nvr : mv) < K) return c;
-    const int64_t rows = cs ? A : (mv + K - 1) / K * V;                 // max slice rows
+    // max slice rows (row split in units of ral V-blocks; the last CTA takes the remainder)
+    const int64_t rows = cs ? A : std::max((mv / ral + K - 1) / K * ral, mv - (mv / ral) * (K - 1) / K * ral) * V;
     const int64_t cvec = cs ? (nvr + K - 1) / K : nvr;                   // max slice vectors per row
     const uint32_t maxw = 256 / V - 1;
     const uint32_t npan = (uint32_t)((cvec + maxw - 1) / maxw);
@@ -1981,6 +1984,7 @@ static RfCfg rf_search(int64_t A, int64_t B, int eb, int device, bool cs, bool c
         }
         c.K = K;
         c.colsplit = cs;
+        c.ralign = cs ? 0 : (uint32_t)ral;
         c.q = q;
         c.npan = npan;
         c.rows_a = (uint32_t)ra;
@@ -2009,9 +2013,20 @@ static RfCfg rf_cfg(int64_t A, int64_t B, int eb, int device) {
     const bool row_first = A * eb / K >= 64;   // as group_choose: row-split pieces >= 64 B
     // the natural split direction first, unchunked configurations before chunked ones
     // (2500 x 5100: column split in one chunk 3.4 TB/s vs row split in chunks 2.8)
+    // Row slices start on 32-byte boundaries of the output rows when that fits
+    // (IPT_TILE_RF_RALIGN, bytes; 0 = any 16-byte V-block boundary): every CTA writes a piece
+    // of every output row, and pieces starting mid-sector made some CTAs' write-out ~40 %
+    // slower (tools/rf_trace.py: exactly the CTAs whose pieces start 16 bytes before a line
+    // boundary), holding up the next tile's group barrier.  C5: 4.40 -> 4.63 TB/s (64 B:
+    // 4.50, 128 B: 4.40 -- coarser units unbalance the slices).
+    const int64_t rab = env_int("IPT_TILE_RF_RALIGN", 32);
+    const int64_t ral = rab > 16 ? rab / 16 : 1;   // V-blocks are 16 bytes of an output row
     RfCfg c;
-    for (int pass = 0; pass < 4 && !c.K; ++pass)
-        c = rf_search(A, B, eb, device, (pass & 1) ? row_first : !row_first, pass >= 2);
+    for (int pass = 0; pass < 4 && !c.K; ++pass) {
+        const bool cs = (pass & 1) ? row_first : !row_first;
+        if (!cs && ral > 1) c = rf_search(A, B, eb, device, cs, pass >= 2, ral);
+        if (!c.K) c = rf_search(A, B, eb, device, cs, pass >= 2, 1);
+    }
     std::lock_guard<std::mutex> lk(mu);
     cache[key] = c;
     return c;
@@ -2057,6 +2072,7 @@ cudaError_t launch_group_rf(const StageDesc &d, TileParams p, const RfCfg &c, vo
     p.rows_a = c.rows_a;
     p.rows_b = c.rows_b;
     p.cpan = c.cpan;
+    p.ralign = c.ralign;
     p.colsplit = c.colsplit ? 1 : 0;
     p.K = (uint32_t)c.K;
     p.nbuf = 1;
@@ -2077,7 +2093,10 @@ cudaError_t launch_group_rf(const StageDesc &d, TileParams p, const RfCfg &c, vo
     }
     const void *kern = nullptr;
     const int rv = std::max(kRfBatch, (c.rv + kRfBatch - 1) / kRfBatch * kRfBatch);
-    const int64_t rbm = (int64_t)(c.colsplit ? d.A : ((d.A / V + c.K - 1) / c.K) * V) - c.rows_a;   // max rows in TMEM
+    const int64_t ral = c.ralign ? c.ralign : 1, mvv = d.A / V;
+    const int64_t rmax = c.colsplit ? d.A
+        : std::max((mvv / ral + c.K - 1) / c.K * ral, mvv - (mvv / ral) * (c.K - 1) / c.K * ral) * V;
+    const int64_t rbm = rmax - (int64_t)c.rows_a;   // max rows in TMEM
     const bool ch = rbm > (int64_t)c.rows_b || c.cpan < c.npan;
 #define IPT_RF(R) if (rv == R) kern = ch ? (const void *)tile_group_rf<EB, R, true> : (const void *)tile_group_rf<EB, R, false>;
     IPT_RF(8) IPT_RF(16) IPT_RF(24) IPT_RF(32)

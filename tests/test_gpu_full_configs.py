@@ -228,6 +228,8 @@ RF_CASES = [  # (M, N, eb, count, stride pad in elements, smem budget override o
     (720, 1800, 4, 5, 0, 20000),       # small tiles forced through the rf path with a small
     (1200, 760, 8, 3, 8, 12000),       # smem budget: TMEM part in several row chunks
     (720, 1800, 4, 2, 0, 60000),       # everything in shared memory (no TMEM part)
+    (4096, 3000, 4, 2, 0, -16),        # row slices on any 16-byte boundary (IPT_TILE_RF_RALIGN=0)
+    (4000, 3200, 4, 2, 0, -64),        # 64-byte aligned row slices
 ]
 
 
@@ -238,8 +240,10 @@ def test_tile_group_rf(monkeypatch, M, N, eb, count, pad, smem):
     (TMA part) and TMEM (tcgen05.st / tcgen05.ld part): every element checked by the
     definition, strided gaps untouched, then transposed back."""
     monkeypatch.setenv("IPT_TILE_RF_FORCE", "1")
-    if smem:
+    if smem > 0:
         monkeypatch.setenv("IPT_TILE_SMEM_MAX", str(smem))
+    elif smem < 0:
+        monkeypatch.setenv("IPT_TILE_RF_RALIGN", str(-smem if smem != -16 else 0))
     dt = torch.int32 if eb == 4 else torch.int64
     stride = M * N + pad
     t = torch.empty(count * stride, dtype=dt, device="cuda")

@@ -36,7 +36,8 @@ if os.environ.get("_CHILD"):
             tot += e0.elapsed_time(e1)
         idx = torch.randint(0, cnt * M * N, (4096,), device="cuda")
         ok = torch.equal(t[idx], seeded.values_torch_sample(idx, eb).to(t.dtype))
-        res[f"{M}x{N}x{eb}b{cnt}"] = (round(2 * M * N * eb * cnt * 6 / (tot / 1e3) / 1e9), kn) if ok else "WRONG"
+        gbs = round(2 * M * N * eb * cnt * 6 / (tot / 1e3) / 1e9)
+        res[f"{M}x{N}x{eb}b{cnt}"] = (gbs, kn) if ok else f"WRONG {gbs}"
         del t
         torch.cuda.empty_cache()
     print(json.dumps(res), flush=True)

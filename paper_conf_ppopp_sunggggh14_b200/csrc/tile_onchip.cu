@@ -74,6 +74,8 @@ struct TileParams {
     uint32_t rows_b;      // tile_group_rf: rows per chunk of the TMEM part
     uint32_t cpan;        // tile_group_rf: panels per chunk of the TMEM part
     uint32_t zero;        // 0 at run time, opaque to the compiler (load-completion dependency)
+    uint32_t gcols;       // tile_group_generic: > 1 = 2-D slice grid, K / gcols row bands x gcols
+                          // column pieces (rank = band * gcols + piece)
 };
 
 __device__ __forceinline__ char *tile_ptr(const TileParams &p, uint64_t t) {
@@ -1051,7 +1053,13 @@ __global__ void __launch_bounds__(512, 1) tile_group_generic(const TileParams p)
     const uint32_t K = p.K;
     const uint32_t rank = blockIdx.x % K;
     uint32_t r0, r1, c0, c1;
-    if (p.colsplit) {
+    if (p.gcols > 1) {   // 2-D grid: output pieces of (m / gr) elements, input pieces n / gc
+        const uint32_t gc = p.gcols, gr = K / gc, ri = rank / gc, ci = rank % gc;
+        r0 = (uint32_t)((uint64_t)ri * p.m / gr);
+        r1 = (uint32_t)((uint64_t)(ri + 1) * p.m / gr);
+        c0 = (uint32_t)((uint64_t)ci * p.n / gc);
+        c1 = (uint32_t)((uint64_t)(ci + 1) * p.n / gc);
+    } else if (p.colsplit) {
         r0 = 0; r1 = p.m;
         c0 = (uint32_t)((uint64_t)rank * p.n / K);
         c1 = (uint32_t)((uint64_t)(rank + 1) * p.n / K);
@@ -1582,6 +1590,7 @@ constexpr long kGroupStaticSmem = 256;   // mbarriers
 
 struct GroupCfg {
     int K = 0, groups = 0, nbuf = 0;
+    int gcols = 0;          // element path: > 1 = 2-D slice grid (K / gcols bands x gcols pieces)
     size_t slice = 0;
     bool colsplit = false;
 };
@@ -1678,13 +1687,102 @@ static GroupCfg group_choose(int64_t A, int64_t B, int eb, uint64_t count, int d
     return g;
 }
 
+// Element path: estimated time of a group configuration, in slice bytes.  Waves x (slice
+// + 4 KB barrier allowance) x a piece factor: every slice is written as pieces of output
+// rows and read as pieces of input rows, and each piece costs ~48 bytes of partial 32-byte
+// sectors at its two ends (fit on 21 stage-2 tiles of the sweep, tools/group_tile_time.py:
+// e.g. 1181 x 1453: column split, 67-byte input pieces 2.44 TB/s -> 4 x 18 grid 4.39);
+// a single slice buffer (no overlap of write-out and fetch) x 1.25.
+static double group_est(const GroupCfg &g, int64_t A, int64_t B, int eb, uint64_t count) {
+    if (!g.K) return 1e300;
+    double out_b, in_b;
+    if (g.gcols > 1) {
+        const int64_t gr = g.K / g.gcols;
+        out_b = (double)((A + gr - 1) / gr * eb);
+        in_b = (double)((B + g.gcols - 1) / g.gcols * eb);
+    } else if (g.colsplit) {
+        out_b = (double)(A * eb);
+        in_b = (double)((B + g.K - 1) / g.K * eb);
+    } else {
+        out_b = (double)((A + g.K - 1) / g.K * eb);
+        in_b = (double)(B * eb);
+    }
+    auto f = [](double pb) { return (pb + 48.0) / pb; };
+    const uint64_t cnt = std::max<uint64_t>(count, 1);
+    const double waves = (double)((cnt + g.groups - 1) / g.groups);
+    return waves * ((double)g.slice + 4096.0) * (0.5 * f(out_b) + 0.5 * f(in_b)) * (g.nbuf == 1 ? 1.25 : 1.0);
+}
+
+// Element path, 2-D slice grid: K = gr x gc CTAs, CTA (band, piece) holds rows
+// [band * A / gr, ..) x columns [piece * B / gc, ..).  For tiles where neither 1-D split
+// gives long pieces on both sides: a row split of a 1279 x 6353 float32 tile writes
+// 34-byte pieces of every output row and its column split does not fit; 4 x 37 writes
+// 1280-byte pieces and reads 172-byte ones (2.86 -> 4.15 TB/s).  Smallest group_est.
+static GroupCfg group_search_2d(int64_t A, int64_t B, int eb, uint64_t count, int device, int nb) {
+    GroupCfg g;
+    const DevProps dp = dev_props(device);
+    const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin);
+    const int V = 16 / eb;
+    const uint64_t cnt = std::max<uint64_t>(count, 1);
+    const int64_t fgr = env_int("IPT_TILE_GROUP_GR", 0);
+    double best = 1e300;
+    for (int64_t gr = 2; gr <= dp.sms / 2; ++gr) {
+        if (fgr && gr != fgr) continue;
+        if (A < gr) break;
+        for (int64_t gc = 2; gr * gc <= dp.sms; ++gc) {
+            if (B < gc) break;
+            const int64_t rows = (A + gr - 1) / gr, L = (B + gc - 1) / gc;
+            size_t slice = (size_t)(rows * (((L + 2 * V - 2) / V) | 1) + 1) * 16;
+            slice = (slice + 127) & ~(size_t)127;
+            if ((long)(nb * slice) + kGroupStaticSmem > budget) continue;
+            GroupCfg c;
+            c.K = (int)(gr * gc);
+            c.gcols = (int)gc;
+            c.groups = (int)std::min<int64_t>(dp.sms / c.K, (int64_t)cnt);
+            c.slice = slice;
+            c.nbuf = nb;
+            const double e = group_est(c, A, B, eb, count);
+            if (e < best * 0.99) {
+                best = e;
+                g = c;
+            }
+        }
+    }
+    return g;
+}
+
 static GroupCfg group_choose_uncached(int64_t A, int64_t B, int eb, uint64_t count, int device, bool generic) {
     const long f = env_int("IPT_TILE_GROUP_COLSPLIT", -1);
-    if (f >= 0) return group_search(A, B, eb, count, device, f != 0, generic);
+    if (f >= 0 && f != 2) return group_search(A, B, eb, count, device, f != 0, generic);
+    const bool grid2d = generic && env_int("IPT_TILE_GROUP_2D", 1);
+    auto search2d = [&]() {
+        GroupCfg g = group_search_2d(A, B, eb, count, device, group_nbuf());
+        if (!g.K && env_int("IPT_TILE_GROUP_SINGLE", 1)) g = group_search_2d(A, B, eb, count, device, 1);
+        return g;
+    };
+    if (f == 2 && grid2d) {   // tests: the 2-D grid whenever one fits
+        const GroupCfg g = search2d();
+        if (g.K) return g;
+    }
     const GroupCfg row = group_search(A, B, eb, count, device, false, generic);
-    if (row.K && A * eb / row.K >= 64) return row;
+    if (!grid2d) {
+        if (row.K && A * eb / row.K >= 64) return row;
+        const GroupCfg col = group_search(A, B, eb, count, device, true, generic);
+        return col.K ? col : row;
+    }
+    // element path: the row split, the column split and the best 2-D grid by group_est
     const GroupCfg col = group_search(A, B, eb, count, device, true, generic);
-    return col.K ? col : row;
+    const GroupCfg g2 = search2d();
+    double er = group_est(row, A, B, eb, count);
+    const double ec = group_est(col, A, B, eb, count), e2 = group_est(g2, A, B, eb, count);
+    // a row split with 16-byte aligned input rows fetches its slices by TMA
+    // (tile_group_tma_elem, ~15 % faster: 9998 x 256 4.38 vs 4.18 TB/s on the 2-D grid)
+    const int V = 16 / eb;
+    if (row.K && (B * eb) % 16 == 0 && env_int("IPT_TILE_GEN_TMAA", 1) &&
+        tma_geom((A + V - 1) / V * V, B, eb, row.K, false).ok)
+        er *= 0.85;
+    if (e2 < er && e2 < ec) return g2;
+    return ec < er ? col : row;
 }
 
 GroupCfg group_cfg(int64_t A, int64_t B, int eb, uint64_t count, int device) {
@@ -1846,8 +1944,9 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
                             cudaStream_t st, int device) {
     if (!ws || !g.K) return cudaErrorInvalidValue;
     if (GENERIC) {
-        const int64_t L = g.colsplit ? (d.B + g.K - 1) / g.K : d.B;
+        const int64_t L = g.gcols > 1 ? (d.B + g.gcols - 1) / g.gcols : g.colsplit ? (d.B + g.K - 1) / g.K : d.B;
         p.q = (uint32_t)(((L + 2 * (16 / EB) - 2) / (16 / EB)) | 1);
+        p.gcols = (uint32_t)std::max(g.gcols, 0);
     } else {
         p.q = fast_q(d.B, d.eb);
     }
@@ -1871,8 +1970,9 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
     CUtensorMap tmap;
     // element path with 16-byte aligned input rows: TMA slices + element write-out
     size_t slice = g.slice;
-    const bool tma_elem = GENERIC && group_tma_setup_elem<EB>(d, p, g, &tmap, &slice, device);
-    const bool tma = tma_elem || (GENERIC ? group_tma_setup_generic<EB>(d, p, g, &tmap)
+    const bool grid2d = g.gcols > 1;   // cp.async slices only
+    const bool tma_elem = GENERIC && !grid2d && group_tma_setup_elem<EB>(d, p, g, &tmap, &slice, device);
+    const bool tma = tma_elem || (GENERIC ? !grid2d && group_tma_setup_generic<EB>(d, p, g, &tmap)
                                           : group_tma_setup<EB>(d, p, g, &tmap));
     cudaError_t e = cudaSuccess;
     if (!p.gexit) {
@@ -1905,8 +2005,8 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     if (env_int("IPT_DEBUG", 0))
-        fprintf(stderr, "[ipt] tile_group%s m=%u n=%u K=%d groups=%d colsplit=%d smem=%zu tiles=%llu\n",
-                GENERIC ? "_generic" : "", p.m, p.n, g.K, g.groups, p.colsplit, g.nbuf * g.slice,
+        fprintf(stderr, "[ipt] tile_group%s m=%u n=%u K=%d groups=%d colsplit=%d gcols=%d nbuf=%d smem=%zu tiles=%llu\n",
+                GENERIC ? "_generic" : "", p.m, p.n, g.K, g.groups, p.colsplit, g.gcols, g.nbuf, g.nbuf * g.slice,
                 (unsigned long long)p.count);
     e = tma ? cudaLaunchKernelEx(&cfg, tkern, p, tmap) : cudaLaunchKernelEx(&cfg, kern, p);
     note_launch();
@@ -2285,6 +2385,7 @@ const char *tile_kernel_name(const StageDesc &d, int device) {
     if (!fast_ok(d) && tile_group_generic_split(d.A, d.B, d.eb, device)) {
         const GroupCfg g = group_cfg_generic(d.A, d.B, d.eb, count, device);
         const int V = 16 / d.eb;
+        if (g.gcols > 1) return "tile_group_generic";   // 2-D grid: cp.async slices
         if (!g.colsplit && (d.B * d.eb) % 16 == 0 && ((uintptr_t)d.base & 15) == 0 && packed &&
             env_int("IPT_TILE_GEN_TMAA", 1) && tma_geom((d.A + V - 1) / V * V, d.B, d.eb, g.K, false).ok)
             return "tile_group_tma_elem";

@@ -778,6 +778,21 @@ def test_ipt_010_group_element_forced_sizes(monkeypatch, K, split):
     assert np.array_equal(to_np(t, 4), oracle_P(a.copy(), batch, A, B, 1, 4)), (K, split)
 
 
+@pytest.mark.parametrize("eb,batch,A,B,gr", [(4, 5, 601, 1203, "0"), (4, 2, 1279, 6353, "0"), (4, 2, 1279, 6353, "8"),
+                                             (4, 3, 2362, 1453, "0"), (8, 2, 1201, 3001, "0"), (8, 2, 3001, 1201, "3"),
+                                             (4, 3, 301, 257, "2"), (4, 2, 1999, 310, "0"), (4, 1, 9797, 103, "0")])
+def test_ipt_010_group_element_grid2d(monkeypatch, eb, batch, A, B, gr):
+    """Element-path group tiles over a 2-D slice grid (gr row bands x gc column pieces, the
+    CTA's piece at its own 16-byte phase): forced for every shape (IPT_TILE_GROUP_COLSPLIT=2),
+    uneven bands and pieces, f64, the sweep's 1279 x 6353 and 2362 x 1453 tiles."""
+    monkeypatch.setenv("IPT_TILE_GROUP_COLSPLIT", "2")
+    monkeypatch.setenv("IPT_TILE_GROUP_GR", gr)
+    a = gen(batch * A * B, eb)
+    t = to_dev(a, eb)
+    ipt.ipt_010_(t, batch, A, B, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, A, B, 1, eb)), (eb, batch, A, B, gr)
+
+
 def test_ipt_010_group_element_misaligned_base():
     """A 16-byte-vectorisable tile at a base that is only 4-byte aligned takes the
     element-path group kernel (any phase)."""

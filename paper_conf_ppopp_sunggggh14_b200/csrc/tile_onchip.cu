@@ -776,10 +776,11 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
         b0 = (uint32_t)((uint64_t)rank * units / K) * ra_;
         b1 = rank + 1 == K ? mv : (uint32_t)((uint64_t)(rank + 1) * units / K) * ra_;
         c0 = 0; c1 = nvr;
-    } else {
+    } else {             // column slices in units of ralign vectors (sector-aligned pieces)
+        const uint32_t ra_ = p.ralign ? p.ralign : 1u, units = nvr / ra_;
         b0 = 0; b1 = mv;
-        c0 = (uint32_t)((uint64_t)rank * nvr / K);
-        c1 = (uint32_t)((uint64_t)(rank + 1) * nvr / K);
+        c0 = (uint32_t)((uint64_t)rank * units / K) * ra_;
+        c1 = rank + 1 == K ? nvr : (uint32_t)((uint64_t)(rank + 1) * units / K) * ra_;
     }
     const uint32_t q = p.q, cvec = c1 - c0;
     const uint32_t rows = (b1 - b0) * V, r0 = b0 * V;
@@ -2032,11 +2033,12 @@ static RfCfg rf_search(int64_t A, int64_t B, int eb, int device, bool cs, bool c
     const DevProps dp = dev_props(device);
     const int K = dp.sms, V = 16 / eb;
     const int64_t mv = A / V, nvr = B / V;
-    if (!cs && (mv % ral || mv / ral < K)) return c;
-    if ((cs ? nvr : mv) < K) return c;
-    // max slice rows (row split in units of ral V-blocks; the last CTA takes the remainder)
-    const int64_t rows = cs ? A : std::max((mv / ral + K - 1) / K * ral, mv - (mv / ral) * (K - 1) / K * ral) * V;
-    const int64_t cvec = cs ? (nvr + K - 1) / K : nvr;                   // max slice vectors per row
+    const int64_t sv = cs ? nvr : mv;   // split dimension in V-blocks / vectors
+    if (sv % ral || sv / ral < K) return c;
+    // max slice (split in units of ral V-blocks / vectors; the last CTA takes the remainder)
+    const int64_t smax = std::max((sv / ral + K - 1) / K * ral, sv - (sv / ral) * (K - 1) / K * ral);
+    const int64_t rows = cs ? A : smax * V;
+    const int64_t cvec = cs ? smax : nvr;                                // max slice vectors per row
     const uint32_t maxw = 256 / V - 1;
     const uint32_t npan = (uint32_t)((cvec + maxw - 1) / maxw);
     const uint32_t q = (uint32_t)(((cvec + npan - 1) / npan) | 1);
@@ -2084,7 +2086,7 @@ static RfCfg rf_search(int64_t A, int64_t B, int eb, int device, bool cs, bool c
         }
         c.K = K;
         c.colsplit = cs;
-        c.ralign = cs ? 0 : (uint32_t)ral;
+        c.ralign = (uint32_t)ral;
         c.q = q;
         c.npan = npan;
         c.rows_a = (uint32_t)ra;
@@ -2110,7 +2112,10 @@ static RfCfg rf_cfg(int64_t A, int64_t B, int eb, int device) {
         if (it != cache.end()) return it->second;
     }
     const int K = dev_props(device).sms;
-    const bool row_first = A * eb / K >= 64;   // as group_choose: row-split pieces >= 64 B
+    // split the longer side (tools/rf_sweep.py per orientation, column vs row split:
+    // 3000 x 4096 4.19 vs 3.99 TB/s, 3200 x 4000 3.33 vs 3.00, 4096 x 3000 3.67 vs 4.85),
+    // and rows only while the row-split pieces are >= 64 B
+    const bool row_first = A >= B && A * eb / K >= 64;
     // the natural split direction first, unchunked configurations before chunked ones
     // (2500 x 5100: column split in one chunk 3.4 TB/s vs row split in chunks 2.8)
     // Row slices start on 32-byte boundaries of the output rows when that fits
@@ -2122,8 +2127,12 @@ static RfCfg rf_cfg(int64_t A, int64_t B, int eb, int device) {
     const int64_t rab = env_int("IPT_TILE_RF_RALIGN", 32);
     const int64_t ral = rab > 16 ? rab / 16 : 1;   // V-blocks are 16 bytes of an output row
     RfCfg c;
+    const long fcs = env_int("IPT_TILE_RF_CS", -1);   // measurement: force the split direction
     for (int pass = 0; pass < 4 && !c.K; ++pass) {
         const bool cs = (pass & 1) ? row_first : !row_first;
+        if (fcs >= 0 && cs != (fcs != 0)) continue;
+        // column slices stay on 16-byte boundaries: 32-byte column units measured slower
+        // (3000 x 4096: 3.97 vs 4.40 TB/s)
         if (!cs && ral > 1) c = rf_search(A, B, eb, device, cs, pass >= 2, ral);
         if (!c.K) c = rf_search(A, B, eb, device, cs, pass >= 2, 1);
     }

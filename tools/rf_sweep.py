@@ -1,7 +1,7 @@
 """Whole-matrix 1-stage plans (m = M, n = N) on batches, timed under env variants:
     SHAPES='[(4096,3000,4,64),(1800,7200,4,1)]' VARIANTS='[{}, {"IPT_TILE_RF_OVERLAP": 0}]' python tools/rf_sweep.py
-prints effective GB/s (2*M*N*b*count / time) per variant and shape, checked against the
-definition on samples."""
+prints effective GB/s (2*M*N*b*count / time) per variant and shape -- both orientations
+together, then M x N and N x M alone -- checked against the definition on samples."""
 import ast
 import json
 import os
@@ -25,6 +25,7 @@ if os.environ.get("_CHILD"):
             ipt.transpose_batched_(t, cnt, N, M, plan_=q)
         flush = torch.zeros(128 << 20, dtype=torch.int32, device="cuda") if M * N * eb * cnt < (200 << 20) else None
         tot = 0.0
+        per = [0.0, 0.0]
         for r in range(6):
             if flush is not None:
                 flush.sum()
@@ -34,10 +35,12 @@ if os.environ.get("_CHILD"):
             e1.record()
             torch.cuda.synchronize()
             tot += e0.elapsed_time(e1)
+            per[r % 2] += e0.elapsed_time(e1)
         idx = torch.randint(0, cnt * M * N, (4096,), device="cuda")
         ok = torch.equal(t[idx], seeded.values_torch_sample(idx, eb).to(t.dtype))
         gbs = round(2 * M * N * eb * cnt * 6 / (tot / 1e3) / 1e9)
-        res[f"{M}x{N}x{eb}b{cnt}"] = (gbs, kn) if ok else f"WRONG {gbs}"
+        fw, bw = (round(2 * M * N * eb * cnt * 3 / (x / 1e3) / 1e9) for x in per)   # M x N, N x M
+        res[f"{M}x{N}x{eb}b{cnt}"] = (gbs, fw, bw, kn) if ok else f"WRONG {gbs}"
         del t
         torch.cuda.empty_cache()
     print(json.dumps(res), flush=True)

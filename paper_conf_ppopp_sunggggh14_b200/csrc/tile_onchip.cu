@@ -63,8 +63,7 @@ struct TileParams {
     uint32_t box_rows;    // tile_group_tma: rows per 2-D TMA box (divides the slice rows)
     uint32_t npan;        // tile_group_tma: column panels per slice (width q vectors each)
     uint32_t pstride;     // tile_group_tma: bytes between panels (128-byte multiple)
-    uint32_t rres;        // tile_group_generic_tma: rows per super-row R (row stride * R % 16 == 0)
-    uint32_t cls_rows;    // tile_group_generic_tma: rows fetched per residue class
+    uint32_t rres;        // tile_group_rf: 1 = 3-D tensor map (strided batch of single tiles)
     int diag;             // group kernels, measurement only (IPT_TILE_DIAG; results invalid):
                           // 1 = no group wait, 2 = no stores, 4 = no loads, 32 = stores
                           // to a second buffer after the data; 16 = timeline
@@ -164,51 +163,6 @@ __device__ __forceinline__ void write_out_pan(const TileParams &p, uint32_t sbas
             rotate_sel<V, E>(col, off);
             stg128_na(g + ((size_t)(bj * V + c) * p.m + (size_t)bi * V) * EB, pack<EB>(col));
         }
-    }
-}
-
-// ------------------------------------------------------------------- TMA ring kernel
-template <int EB>
-__global__ void __launch_bounds__(512) tile_onchip_tma(const TileParams p) {
-    extern __shared__ __align__(128) unsigned char smem[];
-    uint64_t *bar = reinterpret_cast<uint64_t *>(smem);     // up to 8 mbarriers
-    unsigned char *const buf0 = smem + 128;
-    const int tid = threadIdx.x;
-    const int lane = tid & 31;
-    const uint32_t row_bytes = p.n * EB;
-    const uint32_t NB = p.nbuf;
-
-    if (tid == 0) {
-        for (uint32_t b = 0; b < NB; ++b) mbar_init(&bar[b], 1);
-        fence_mbar_init();
-    }
-    __syncthreads();
-
-    auto issue = [&](uint64_t t, uint32_t b) {   // warp 0 only
-        const char *g = tile_ptr(p, t);
-        if (lane == 0) mbar_arrive_expect_tx(&bar[b], (uint32_t)p.tile_bytes);
-        __syncwarp();
-        unsigned char *dst = buf0 + (size_t)b * p.buf_bytes;
-        for (uint32_t i = lane; i < p.m; i += 32)
-            bulk_g2s(dst + (size_t)i * p.q * 16, g + (size_t)i * row_bytes, row_bytes, &bar[b]);
-    };
-
-    // prologue: NB - 1 tiles in flight
-    if (tid < 32) {
-        for (uint32_t j = 0; j + 1 < NB; ++j) {
-            const uint64_t t = blockIdx.x + (uint64_t)j * gridDim.x;
-            if (t < p.count) issue(t, j);
-        }
-    }
-    uint32_t it = 0;
-    for (uint64_t t = blockIdx.x; t < p.count; t += gridDim.x, ++it) {
-        const uint32_t b = it % NB;
-        const uint64_t tn = t + (uint64_t)(NB - 1) * gridDim.x;
-        // buffer (it + NB - 1) % NB was consumed in iteration it - 1 (barrier below)
-        if (tn < p.count && tid < 32) issue(tn, (it + NB - 1) % NB);
-        mbar_wait(&bar[b], (it / NB) & 1);
-        write_out<EB>(p, smem_u32(buf0) + b * p.buf_bytes, tile_ptr(p, t));
-        __syncthreads();
     }
 }
 
@@ -1133,111 +1087,6 @@ __global__ void __launch_bounds__(512, 1) tile_group_generic(const TileParams p)
     group_loop(p, s0, mbar, load, write);
 }
 
-// ------------------------------------------- group-split element-path kernel, TMA slices
-// Element-path tiles (sides not multiples of 16/elem) whose slices are fetched by 2-D TMA
-// boxes.  A tensor map needs 16-byte row strides, so rows are grouped R at a time into
-// super-rows (R = 16 / gcd(n * elem, 16), a tensor of (count*m/R) super-rows x R*n
-// elements; requires m % R == 0): slice row i of residue class s = i % R is super-row
-// row-of-(first row of the class) + i / R, column offset ((G0 + s) % R) * n.  Each class
-// lands in its own region (128-byte aligned), rows at an odd pitch of q vectors; boxes
-// start 16-byte aligned, so a class's rows sit at a phase sh < 16/elem and the write-out
-// realigns two vectors per element group as tile_group_generic does.  Boxes may read rows
-// or columns beyond the slice (same tile, the next tile, or out of bounds -> zero) into
-// padding that is never written out.  Write-out as tile_group_generic, with the lanes of
-// a warp grouped by residue class so each 8-lane phase of an LDS.128 reads 8 consecutive
-// rows of one class (conflict-free); the warp still stores 32 consecutive output elements.
-template <int EB>
-__global__ void __launch_bounds__(512, 1) tile_group_generic_tma(const TileParams p, const __grid_constant__ CUtensorMap tmap) {
-    constexpr uint32_t PV = 16 / EB;
-    using E = typename Elem<EB>::T;
-    extern __shared__ __align__(128) unsigned char smem[];
-    const uint32_t s0 = smem_u32(smem);
-    const uint32_t K = p.K;
-    const uint32_t rank = blockIdx.x % K;
-    uint32_t r0, r1, c0, c1;
-    if (p.colsplit) {
-        r0 = 0; r1 = p.m;
-        c0 = (uint32_t)((uint64_t)rank * p.n / K);
-        c1 = (uint32_t)((uint64_t)(rank + 1) * p.n / K);
-    } else {
-        c0 = 0; c1 = p.n;
-        r0 = (uint32_t)((uint64_t)rank * p.m / K);
-        r1 = (uint32_t)((uint64_t)(rank + 1) * p.m / K);
-    }
-    const uint32_t rows = r1 - r0, L = c1 - c0, Q = p.q, R = p.rres, H = p.cls_rows;
-    const uint32_t cstride = p.pstride;                    // bytes per (panel, class) region
-    const FastDiv32 divq = make_fastdiv32_dev(Q);
-    constexpr uint32_t CH = 8;                            // column blocks per write task
-    const uint32_t nrb = (rows + 31) / 32, ncb = (L + PV - 1) / PV, nch = (ncb + CH - 1) / CH;
-    const uint32_t ntask = nrb * nch;
-    const FastDiv32 divrb = make_fastdiv32_dev(nrb);
-    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
-    const uint64_t mEB = (uint64_t)p.m * EB;
-    const uint32_t lpc = 32 / R;                          // lanes per residue class
-    const uint32_t lcls = lane / lpc, lj = lane % lpc;
-    __shared__ __align__(8) uint64_t mbar[kGroupMaxBuf];
-
-    auto load = [&](const char *g, uint32_t sb) {
-        if (threadIdx.x != 0) return;
-        const uint64_t G0 = (uint64_t)(g - p.base) / ((uint64_t)p.n * EB) + r0;
-        uint64_t *bar = &mbar[(sb - s0) / p.buf_bytes];
-        mbar_expect_tx(bar, p.npan * R * H * Q * 16);
-        const uint32_t sbar = smem_u32(bar);
-        for (uint32_t pn = 0; pn < p.npan; ++pn)
-            for (uint32_t c = 0; c < R; ++c) {
-                const uint64_t Gs = G0 + c;
-                // box starts 16-byte aligned: the class's first element lands at phase sh
-                const uint32_t xe = (uint32_t)((Gs % R) * p.n + c0);
-                const int32_t x = (int32_t)((xe & ~(PV - 1)) + pn * Q * PV);
-                const uint32_t dst = sb + (pn * R + c) * cstride;
-                for (uint32_t r = 0; r < H; r += p.box_rows)
-                    tma_load_2d(dst + r * Q * 16, &tmap, x, (int32_t)(Gs / R + r), sbar);
-            }
-    };
-    auto write = [&](char *g, uint32_t sb, auto probe) {
-        for (uint32_t task = warp; task < ntask; task += nw) {
-            probe();
-            uint32_t ch, rb;
-            fdivmod32(task, divrb, ch, rb);
-            const uint32_t i = rb * 32 + lj * R + lcls;          // i % R == lcls
-            if (i >= rows) continue;
-            const uint32_t srow = sb + lcls * cstride + (i / R) * Q * 16;
-            const uint32_t sh = ((((r0 + lcls) % R) * p.n + c0) & (PV - 1));   // class phase
-            const uint32_t cfirst = ch * CH * PV;
-            char *out = g + ((uint64_t)(c0 + cfirst) * p.m + r0 + i) * EB;
-#pragma unroll 2
-            for (uint32_t cbl = 0; cbl < CH; ++cbl) {
-                const uint32_t c = cfirst + cbl * PV;
-                if (c >= L) break;
-                const uint32_t w = sh + c, v = w / PV, o = w % PV;
-                uint32_t pn, pv;
-                fdivmod32(v, divq, pn, pv);
-                const uint32_t a0 = srow + pn * R * cstride + pv * 16;
-                const uint32_t a1 = (pv + 1 == Q) ? srow + (pn + 1) * R * cstride : a0 + 16;
-                E x[2 * PV];
-                {
-                    E ex[PV], ey[PV];
-                    unpack<EB>(lds128(a0), ex);
-                    unpack<EB>(lds128(a1), ey);
-#pragma unroll
-                    for (uint32_t k = 0; k < PV; ++k) { x[k] = ex[k]; x[PV + k] = ey[k]; }
-                }
-#pragma unroll
-                for (uint32_t sft = 1; sft < PV; sft <<= 1) {   // x[k] <- x[k + o]
-                    const bool f = (o & sft) != 0;
-#pragma unroll
-                    for (uint32_t k = 0; k + sft < 2 * PV; ++k) x[k] = f ? x[k + sft] : x[k];
-                }
-                char *oc = out + (uint64_t)cbl * PV * mEB;
-#pragma unroll
-                for (uint32_t k = 0; k < PV; ++k)
-                    if (c + k < L) *reinterpret_cast<E *>(oc + k * mEB) = x[k];
-            }
-        }
-    };
-    group_loop(p, s0, mbar, load, write);
-}
-
 // ------------------------------------------------------------------- generic kernel
 // Any element size and any m x n that fits (Fig. 1 for a CUDA block).  The tile is
 // contiguous, so when it is 16-byte aligned it is loaded with 16-byte vectors; elements
@@ -1385,17 +1234,10 @@ __global__ void __launch_bounds__(512, 1) tile_generic_cluster(const TileParams 
 // ------------------------------------------------------------------------ host side
 namespace {
 
-enum { MODE_LDG = 0, MODE_TMA = 1 };
-
-int tile_mode() { return (int)env_int("IPT_TILE_MODE", MODE_LDG); }
 int tile_threads(uint64_t tile_bytes) {
     // small tiles: 256 threads (fewer idle threads in the write-out), else 512
     long t = env_int("IPT_TILE_THREADS", tile_bytes < 48 * 1024 ? 256 : 512);
     return (t == 256 || t == 512) ? (int)t : 512;
-}
-uint32_t tma_nbuf() {
-    long b = env_int("IPT_TILE_STAGES", 2);
-    return (uint32_t)(b < 2 ? 2 : (b > 8 ? 8 : b));
 }
 
 bool vec_ok(int64_t A, int64_t B, int eb) {
@@ -1418,9 +1260,7 @@ uint32_t fast_q(int64_t B, int eb) {
 }
 
 size_t fast_smem(int64_t A, int64_t B, int eb) {
-    const size_t buf = (size_t)A * fast_q(B, eb) * 16;
-    if (tile_mode() == MODE_TMA) return 128 + tma_nbuf() * buf;
-    return buf;
+    return (size_t)A * fast_q(B, eb) * 16;
 }
 
 uint32_t generic_pitch(int64_t B) {
@@ -1540,45 +1380,6 @@ static TmaGeom tma_geom(int64_t A, int64_t B, int eb, int K, bool cs) {
     return t;
 }
 
-// Slice geometry of tile_group_generic_tma (element path): R rows per super-row, H rows
-// fetched per residue class (boxes of br rows), npan column panels of q vectors.
-struct TmaGeomG {
-    bool ok = false;
-    uint32_t R = 0, H = 0, q = 0, npan = 0, br = 0;
-    size_t cstride = 0, bytes = 0;
-};
-
-// Opt-in (IPT_TILE_GROUP_TMA_GENERIC=1): measured slower than the cp.async element slices
-// on 7 of 8 panel shapes (e.g. 14803x256 4.98 -> 4.39 TB/s; 9998x128 4.94 -> 5.17): the
-// element path is bound by its 4-byte-store write-out, not by its loads.
-static TmaGeomG tma_geom_generic(int64_t A, int64_t B, int eb, int K, bool cs) {
-    TmaGeomG t;
-    if ((eb != 4 && eb != 8) || !env_int("IPT_TILE_GROUP_TMA", 1) ||
-        !env_int("IPT_TILE_GROUP_TMA_GENERIC", 0))
-        return t;
-    const uint32_t PV = 16 / eb;
-    const int64_t rowb = B * eb;
-    int64_t g = 16;
-    while (rowb % g) g >>= 1;                      // gcd(rowb, 16)
-    t.R = (uint32_t)(16 / g);
-    if (A % t.R) return t;
-    const int64_t L = cs ? (B + K - 1) / K : B;
-    const int64_t rows = cs ? A : (A + K - 1) / K;
-    t.H = (uint32_t)((rows + t.R - 1) / t.R);
-    // vectors per row: the slice row at phase < PV, plus the second vector the write-out's
-    // aligner reads after the last element
-    const uint32_t need = (uint32_t)((L + 2 * PV - 2) / PV + 1);
-    const uint32_t maxw = 256 / PV - 1;
-    t.npan = (need + maxw - 1) / maxw;
-    t.q = ((need + t.npan - 1) / t.npan) | 1u;
-    for (uint32_t b = std::min<uint32_t>(t.H, 256); b >= 1; --b)
-        if (t.H % b == 0 && (b == t.H || b % 8 == 0)) { t.br = b; break; }
-    if (t.br == 0 || (t.br < 16 && t.br != t.H)) return t;
-    t.cstride = (((size_t)t.H * t.q * 16) + 127) & ~(size_t)127;
-    t.bytes = (size_t)t.npan * t.R * t.cstride;
-    t.ok = true;
-    return t;
-}
 
 // Group split (tile_group_db / tile_group_generic): K CTAs per tile, `groups` tiles in
 // flight, nbuf slice buffers per CTA.  K minimises waves x (slice + 4 KB barrier
@@ -1647,8 +1448,6 @@ static GroupCfg group_search_nb(int64_t A, int64_t B, int eb, uint64_t count, in
             const TmaGeom t = tma_geom(A, B, eb, K, cs);
             if (t.ok) slice = std::max(slice, t.bytes);
         } else {
-            const TmaGeomG t = tma_geom_generic(A, B, eb, K, cs);
-            if (t.ok) slice = std::max(slice, t.bytes);
             if (!cs && (B * eb) % 16 == 0 && env_int("IPT_TILE_GEN_TMAA", 1)) {   // tile_group_tma_elem
                 const TmaGeom te = tma_geom((A + V - 1) / V * V, B, eb, K, false);
                 if (te.ok) slice = std::max(slice, te.bytes);
@@ -1881,38 +1680,6 @@ bool group_tma_setup_elem(const StageDesc &d, TileParams &p, const GroupCfg &g, 
     return true;
 }
 
-template <int EB>
-bool group_tma_setup_generic(const StageDesc &d, TileParams &p, const GroupCfg &g, CUtensorMap *tm) {
-    if (EB != 4 && EB != 8) return false;
-    if (d.outer > 1 && d.ostride != d.inner * (int64_t)p.tile_bytes) return false;
-    if (((uintptr_t)d.base & 15) != 0) return false;
-    const TmaGeomG t = tma_geom_generic(d.A, d.B, EB, g.K, g.colsplit);
-    if (!t.ok || t.bytes > g.slice) return false;
-    auto enc = tensor_map_encoder();
-    if (!enc) return false;
-    const uint64_t total_rows = (uint64_t)(d.outer * d.inner) * (uint64_t)d.A;
-    cuuint64_t dims[2] = {(cuuint64_t)(d.B * t.R), (cuuint64_t)(total_rows / t.R)};
-    cuuint64_t strides[1] = {(cuuint64_t)(d.B * t.R * EB)};
-    cuuint32_t box[2] = {t.q * (16 / EB), t.br};
-    cuuint32_t estr[2] = {1, 1};
-    CUresult r = enc(tm, EB == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 2, d.base,
-                     dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    if (r != CUDA_SUCCESS) {
-        if (env_int("IPT_DEBUG", 0)) fprintf(stderr, "[ipt] tensor map encode failed (%d)\n", (int)r);
-        return false;
-    }
-    p.q = t.q;
-    p.npan = t.npan;
-    p.rres = t.R;
-    p.cls_rows = t.H;
-    p.box_rows = t.br;
-    p.pstride = (uint32_t)t.cstride;
-    if (env_int("IPT_DEBUG", 0))
-        fprintf(stderr, "[ipt] tile_group_generic_tma R=%u H=%u q=%u npan=%u box=%ux%u\n", t.R, t.H, t.q,
-                t.npan, t.q * (16 / EB), t.br);
-    return true;
-}
 
 // Library-owned group counters per (device, stream): arrivals (kTileWsBytes) then per-group
 // exit counters (kTileWsBytes), zeroed once ON that stream, re-zeroed by each launch's last
@@ -1973,8 +1740,7 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
     size_t slice = g.slice;
     const bool grid2d = g.gcols > 1;   // cp.async slices only
     const bool tma_elem = GENERIC && !grid2d && group_tma_setup_elem<EB>(d, p, g, &tmap, &slice, device);
-    const bool tma = tma_elem || (GENERIC ? !grid2d && group_tma_setup_generic<EB>(d, p, g, &tmap)
-                                          : group_tma_setup<EB>(d, p, g, &tmap));
+    const bool tma = tma_elem || (!GENERIC && group_tma_setup<EB>(d, p, g, &tmap));
     cudaError_t e = cudaSuccess;
     if (!p.gexit) {
         e = cudaMemsetAsync(ws, 0, (size_t)g.groups * g.nbuf * kGroupCtrStride, st);
@@ -1993,7 +1759,7 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
         }
     };
     set_smem((const void *)kern);
-    auto tkern = tma_elem ? tile_group_tma_elem<EB> : (GENERIC ? tile_group_generic_tma<EB> : tile_group_tma<EB>);
+    auto tkern = tma_elem ? tile_group_tma_elem<EB> : tile_group_tma<EB>;
     if (tma) set_smem((const void *)tkern);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)(g.groups * g.K), 1, 1);
@@ -2380,9 +2146,9 @@ const char *tile_kernel_name(const StageDesc &d, int device) {
         return "tile_group_rf";
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) <= budget) {
         const size_t smem = fast_smem(d.A, d.B, d.eb);
-        if (smem > 113 * 1024 && env_int("IPT_TILE_STREAM", 1) && tile_mode() != MODE_TMA)
+        if (smem > 113 * 1024 && env_int("IPT_TILE_STREAM", 1))
             return "tile_onchip_stream";
-        return tile_mode() == MODE_TMA ? "tile_onchip_tma" : "tile_onchip_ldg";
+        return "tile_onchip_ldg";
     }
     const uint64_t count = (uint64_t)(d.outer * d.inner);
     const bool packed = d.outer <= 1 || d.ostride == d.inner * d.A * d.B * d.eb;
@@ -2398,8 +2164,7 @@ const char *tile_kernel_name(const StageDesc &d, int device) {
         if (!g.colsplit && (d.B * d.eb) % 16 == 0 && ((uintptr_t)d.base & 15) == 0 && packed &&
             env_int("IPT_TILE_GEN_TMAA", 1) && tma_geom((d.A + V - 1) / V * V, d.B, d.eb, g.K, false).ok)
             return "tile_group_tma_elem";
-        const TmaGeomG t = tma_geom_generic(d.A, d.B, d.eb, g.K, g.colsplit);
-        return (packed && t.ok && t.bytes <= g.slice) ? "tile_group_generic_tma" : "tile_group_generic";
+        return "tile_group_generic";
     }
     if (fast_ok(d) && (long)fast_smem(d.A, d.B, d.eb) > budget && tile_cluster_k(d.A, d.B, d.eb, device))
         return "tile_onchip_cluster";
@@ -2450,10 +2215,9 @@ cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, in
         p.divNV = make_fastdiv((uint64_t)(d.B / V));
         p.divNV32 = make_fastdiv32((uint32_t)(d.B / V));
         p.divMV32 = make_fastdiv32((uint32_t)(d.A / V));
-        p.nbuf = tma_nbuf();
         const size_t smem = fast_smem(d.A, d.B, d.eb);
         const bool big = smem > 113 * 1024 && env_int("IPT_TILE_BIGU", 1);
-        if (smem > 113 * 1024 && env_int("IPT_TILE_STREAM", 1) && tile_mode() != MODE_TMA) {
+        if (smem > 113 * 1024 && env_int("IPT_TILE_STREAM", 1)) {
             p.K = 1;
             p.colsplit = 0;
             switch (d.eb) {
@@ -2462,22 +2226,14 @@ cudaError_t launch_tile_onchip(const StageDesc &d, void *ws, cudaStream_t st, in
                 case 16: return go(tile_onchip_stream<16>, p, smem, st, device);
             }
         }
-        if (tile_mode() == MODE_TMA) {
-            switch (d.eb) {
-                case 4: return go(tile_onchip_tma<4>, p, smem, st, device);
-                case 8: return go(tile_onchip_tma<8>, p, smem, st, device);
-                case 16: return go(tile_onchip_tma<16>, p, smem, st, device);
-            }
-        } else {
-            switch (d.eb) {
-                // one CTA per SM for > 113 KB: twice the loads in flight per thread
-                case 4: return big ? go(tile_onchip_ldg<4, 16, 1>, p, smem, st, device)
-                                   : go(tile_onchip_ldg<4, 8>, p, smem, st, device);
-                case 8: return big ? go(tile_onchip_ldg<8, 16, 1>, p, smem, st, device)
-                                   : go(tile_onchip_ldg<8, 8>, p, smem, st, device);
-                case 16: return big ? go(tile_onchip_ldg<16, 16, 1>, p, smem, st, device)
-                                    : go(tile_onchip_ldg<16, 8>, p, smem, st, device);
-            }
+        switch (d.eb) {
+            // one CTA per SM for > 113 KB: twice the loads in flight per thread
+            case 4: return big ? go(tile_onchip_ldg<4, 16, 1>, p, smem, st, device)
+                               : go(tile_onchip_ldg<4, 8>, p, smem, st, device);
+            case 8: return big ? go(tile_onchip_ldg<8, 16, 1>, p, smem, st, device)
+                               : go(tile_onchip_ldg<8, 8>, p, smem, st, device);
+            case 16: return big ? go(tile_onchip_ldg<16, 16, 1>, p, smem, st, device)
+                                : go(tile_onchip_ldg<16, 8>, p, smem, st, device);
         }
     }
     if (fast_ok(d) && tile_group_split(d.A, d.B, d.eb, device)) {

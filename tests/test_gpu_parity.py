@@ -692,10 +692,9 @@ def test_ipt_010_group_tma_slices(monkeypatch, tma, eb, batch, A, B, K):
 @pytest.mark.parametrize("eb,batch,A,B,K", [(4, 2, 128, 9998, "0"), (4, 2, 9998, 128, "0"), (4, 1, 256, 14803, "0"),
                                             (4, 1, 14803, 256, "0"), (4, 2, 192, 9998, "0"), (4, 3, 601, 1203, "5"),
                                             (8, 2, 3001, 62, "0"), (8, 2, 62, 3001, "7"), (4, 2, 1998, 130, "9")])
-def test_ipt_010_group_tma_element_slices(monkeypatch, eb, batch, A, B, K):
-    """Element-path group tiles with TMA slices (opt-in path): rows grouped R = 1, 2, 4 per
-    super-row, per-class phases realigned on write-out, one or two panels."""
-    monkeypatch.setenv("IPT_TILE_GROUP_TMA_GENERIC", "1")
+def test_ipt_010_group_element_slices_forced_k(monkeypatch, eb, batch, A, B, K):
+    """Element-path group tiles whose rows are 4- or 8-byte but not 16-byte aligned
+    (row pieces at any 16-byte phase), forced group sizes, one or two slice buffers."""
     monkeypatch.setenv("IPT_TILE_GROUP_K", K)
     a = gen(batch * A * B, eb)
     t = to_dev(a, eb)
@@ -810,11 +809,11 @@ SQ_SIDES = [2, 3, 7, 15, 16, 17, 63, 64, 65, 100, 127, 128, 129, 255, 256, 257, 
 
 
 @pytest.mark.parametrize("eb", [1, 2, 4, 8, 16])
-@pytest.mark.parametrize("path", ["auto", "tma", "vec", "elem", "elem_pf32", "elem_pf64", "elem_plain", "tb512",
+@pytest.mark.parametrize("path", ["auto", "vec", "elem", "elem_pf32", "elem_pf64", "elem_plain", "tb512",
                                   "tb512nt512", "swz", "swz512", "noswz"])
 def test_square_swap_sides(monkeypatch, eb, path):
-    """ipt_010 on square items through the swap kernel (TMA ring by default, register
-    staged, element path): every side spans ragged block edges (g not a multiple of the
+    """ipt_010 on square items through the swap kernel (register-staged 16-byte path,
+    element path): every side spans ragged block edges (g not a multiple of the
     block) and, for g % (16/b) != 0, the element path; batches fold several items into
     one launch (rows of a ragged last block belong to the next item)."""
     monkeypatch.setenv("IPT_SQ_FORCE", "1")
@@ -826,10 +825,6 @@ def test_square_swap_sides(monkeypatch, eb, path):
         monkeypatch.setenv("IPT_SQ_TB", "512")
     if path == "tb512nt512":
         monkeypatch.setenv("IPT_SQ_NT", "512")
-    if path in ("vec", "tb512", "tb512nt512"):
-        monkeypatch.setenv("IPT_SQ_TMA", "0")
-    if path == "tma":
-        monkeypatch.setenv("IPT_SQ_TMA", "1")
     if path.startswith("swz"):
         monkeypatch.setenv("IPT_SQ_SWZ", "1")
         monkeypatch.setenv("IPT_SQ_TB", "512" if path == "swz512" else "256")
@@ -918,25 +913,8 @@ def test_square_host_path():
     assert np.array_equal(h.numpy().view(np.uint32), oracle.transpose_inplace(a.copy(), M, M))
 
 
-@pytest.mark.parametrize("nb,st,tma", [(2, 0, 1), (3, 2, 1), (7, 1, 1), (0, 3, 1), (0, 2, 0),
-                                       (0, 1, 0), (0, 0, 0)])
-def test_square_swap_tma_ring_depths(monkeypatch, nb, st, tma):
-    """The TMA ring wraps many times (phase parity of full/empty barriers) at small depths;
-    super-tile pair orders (S = 2^st, empty slots below the diagonal and past the edge)
-    on both the TMA and the register-staged kernels."""
-    monkeypatch.setenv("IPT_SQ_FORCE", "1")
-    monkeypatch.setenv("IPT_SQ_NB", str(nb))
-    monkeypatch.setenv("IPT_SQ_ST", str(st))
-    monkeypatch.setenv("IPT_SQ_TMA", str(tma))
-    for (batch, g, eb) in [(3, 1000, 4), (2, 777 * 2, 8), (40, 129, 4), (5, 96, 16)]:
-        a = gen(batch * g * g, eb)
-        t = to_dev(a, eb)
-        ipt.ipt_010_(t, batch, g, g, elem_bytes=eb)
-        assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), batch, g, g, 1, eb)), (batch, g, eb)
-
-
-def test_square_swap_strided_batch_tma(monkeypatch):
-    """3-D tensor map: outer items at a stride (a gap after every item) -- gaps untouched."""
+def test_square_swap_strided_batch(monkeypatch):
+    """Outer items at a stride (a gap after every item) -- gaps untouched."""
     count, M, gap = 4, 1000, 4 * 7
     stride = M * M + gap
     a = gen(count * stride, 4)

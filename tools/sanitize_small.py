@@ -37,7 +37,7 @@ def sq(g, batch, eb, env):
         del os.environ[k]
 for env in [{"IPT_SQ_FORCE": "1", "IPT_SQ_TB": "256"}, {"IPT_SQ_FORCE": "1", "IPT_SQ_TB": "512"},
             {"IPT_SQ_FORCE": "1", "IPT_SQ_TB": "512", "IPT_SQ_NT": "512"},
-            {"IPT_SQ_FORCE": "1", "IPT_SQ_ELEM": "1"}, {"IPT_SQ_FORCE": "1", "IPT_SQ_TMA": "1"}]:
+            {"IPT_SQ_FORCE": "1", "IPT_SQ_ELEM": "1"}]:
     sq(300, 2, 4, env)
     sq(129, 3, 8, env)
 # element-path group tiles: TMA slices (aligned input rows) and cp.async slices

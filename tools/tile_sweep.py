@@ -1,4 +1,4 @@
-"""Microbenchmark of the tile stage (0010!) alone across modes / tile shapes."""
+"""Microbenchmark of the tile stage (0010!) alone across tile shapes (THREADS=256|512)."""
 import os, sys, itertools, json
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
@@ -20,12 +20,12 @@ def bench(m, n, reps=5):
     return 2 * cnt * m * n * 4 / (ms / 1e3) / 1e9
 import ast
 shapes = ast.literal_eval(os.environ.get("SHAPES", "[(128, 200)]"))
-for mode, thr, st in [("0", "512", "2")]:
-    os.environ["IPT_TILE_MODE"] = mode; os.environ["IPT_TILE_THREADS"] = thr; os.environ["IPT_TILE_STAGES"] = st
-    res = {}
-    for (m, n) in shapes:
-        try:
-            res[f"{m}x{n}"] = round(bench(m, n), 0)
-        except Exception as e:
-            res[f"{m}x{n}"] = str(e)[:40]
-    print(f"mode={'ldg' if mode=='0' else 'tma'} threads={thr} stages={st}", json.dumps(res), flush=True)
+thr = os.environ.get("THREADS", "512")
+os.environ["IPT_TILE_THREADS"] = thr
+res = {}
+for (m, n) in shapes:
+    try:
+        res[f"{m}x{n}"] = round(bench(m, n), 0)
+    except Exception as e:
+        res[f"{m}x{n}"] = str(e)[:40]
+print(f"threads={thr}", json.dumps(res), flush=True)

@@ -285,8 +285,20 @@ def run_reference(args, world, rank):
         "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
-    print(json.dumps(line), flush=True)
+    emit(line, args)
     return 0
+
+
+def emit(line, args):
+    """Print the bench line; with --record, append it to a JSONL run record as well."""
+    print(json.dumps(line), flush=True)
+    if getattr(args, "record", None):
+        rev = subprocess.run(["git", "rev-parse", "--short", "HEAD"], capture_output=True, text=True,
+                             cwd=os.path.dirname(os.path.abspath(__file__))).stdout.strip()
+        rec = dict(line, recorded_utc=time.strftime("%Y-%m-%dT%H:%M:%SZ", time.gmtime()),
+                   git_rev=rev or None, argv=sys.argv[1:])
+        with open(args.record, "a") as f:
+            f.write(json.dumps(rec) + "\n")
 
 
 # ---------------------------------------------------------------------- ours: common
@@ -465,6 +477,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--record", default=os.environ.get("IPT_BENCH_RECORD"),
+                    help="also append the JSON line, with a UTC timestamp and the git revision, "
+                         "to this JSONL run-record file")
     args = ap.parse_args()
 
     # --gpus N outside torchrun: re-launch under torch.distributed.run, one rank per GPU
@@ -714,7 +729,7 @@ def main():
             "per_shape": per_shape, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches, "clocks": clk, "verified": ok, "sub": subs,
         }
-        print(json.dumps(line), flush=True)
+        emit(line, args)
     part.barrier()
     if world > 1:
         import torch.distributed as dist

@@ -7,6 +7,7 @@
 //   stage 3  0100! P(count*N', M', n, m)       -> cycle_global  (or identity)
 // The batch is folded into every stage (the instances are independent), so each
 // stage is a single launch regardless of `count`.
+#include <nvtx3/nvToolsExt.h>
 #include "ipt_internal.h"
 
 #include <cstdio>
@@ -350,7 +351,14 @@ ipt_status run_plan(char *base, int64_t count, int64_t stride, const ipt_plan_t 
     plan_stages(p, base, count, stride, sd);
     rec(events, 0, st);
     cudaError_t e = cudaSuccess;
+    // NVTX range per launched stage (header-only NVTX3: a no-op unless a profiler injects
+    // itself): nsys/ncu timelines and `ncu --nvtx --nvtx-include "ipt 0010!/"` filters
+    static const char *const kStageNames[3] = {"ipt 100! (stage 1)", "ipt 0010! (stage 2)",
+                                               "ipt 0100! (stage 3)"};
+    const bool nvtx = env_int("IPT_NVTX", 1) != 0;
     for (int i = 0; i < 3 && e == cudaSuccess; ++i) {
+        const bool ranged = nvtx && p->variant[i] != IPT_VAR_IDENTITY;
+        if (ranged) nvtxRangePushA(kStageNames[i]);
         switch (p->variant[i]) {
             case IPT_VAR_IDENTITY: break;
             case IPT_VAR_TILE_ONCHIP: e = launch_tile_onchip(sd[i], ws, st, device); break;
@@ -358,6 +366,7 @@ ipt_status run_plan(char *base, int64_t count, int64_t stride, const ipt_plan_t 
             case IPT_VAR_CYCLE_GLOBAL: e = launch_cycle_global(sd[i], ws, st, device); break;
             default: e = cudaErrorInvalidValue; break;
         }
+        if (ranged) nvtxRangePop();
         if (e == cudaSuccess) rec(events, i + 1, st);
     }
     return cuda_status(release_ws(w, st, e));

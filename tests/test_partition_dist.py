@@ -92,18 +92,24 @@ def test_two_rank_gloo_bench_bookkeeping(count):
         assert abs(gbs - job * 3 / 0.020 / 1e9) < 1e-9
 
 
-def test_bench_gpus_flag_spawns_ranks():
+def test_bench_gpus_flag_spawns_ranks(tmp_path):
     """`bench.py --gpus 2` without WORLD_SIZE re-launches itself with 2 ranks; each rank
     checks WORLD_SIZE == --gpus (here under the reference arm, which needs no GPU: rank 0
     prints the line, the other rank exits 0)."""
     env = dict(os.environ)
     env.pop("WORLD_SIZE", None)
+    record = os.path.join(str(tmp_path), "runs.jsonl")
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--impl",
-                        "reference", "--steps", "1", "--warmup", "0"],
+                        "reference", "--steps", "1", "--warmup", "0", "--record", record],
                        capture_output=True, text=True, timeout=600, env=env, cwd=ROOT)
     assert r.returncode == 0, r.stderr[-2000:]
     lines = [x for x in r.stdout.splitlines() if x.startswith("{")]
     assert len(lines) == 1 and '"n_gpus": 2' in lines[0] and '"impl": "reference"' in lines[0]
+    # --record: the same line (rank 0 only) appended to a JSONL run record, stamped
+    import json
+    recs = [json.loads(x) for x in open(record)]
+    assert len(recs) == 1 and recs[0]["value"] == json.loads(lines[0])["value"]
+    assert recs[0]["recorded_utc"].endswith("Z") and "--record" in recs[0]["argv"]
     # a mismatched rank count is refused
     env.update(WORLD_SIZE="1", RANK="0", LOCAL_RANK="0")
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2"],

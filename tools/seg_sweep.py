@@ -36,7 +36,7 @@ if os.environ.get("_CHILD"):
     print(json.dumps(res), flush=True)
 else:
     extra = json.loads(os.environ.get("VARIANTS", "[{}]"))
-    for mode in ["0", "2"]:
+    for mode in json.loads(os.environ.get("MODES", "[\"0\", \"2\"]")):
         for v in extra:
             env = dict(os.environ, _CHILD="1", IPT_CYC_SEG=mode, **{k: str(x) for k, x in v.items()})
             out = subprocess.run([sys.executable, __file__], env=env, capture_output=True, text=True)

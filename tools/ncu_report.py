@@ -1,6 +1,6 @@
 """Summarise ncu --set full captures (gpurun_out/<name>.ncu-rep) into a markdown table.
 
-    python tools/ncu_report.py <out.md> name:algorithmic_bytes:units:description ...
+    python tools/ncu_report.py <out.md> name[@k]:algorithmic_bytes:units:description ...
 
 For each capture: duration, DRAM read / write against the algorithmic bytes (read + write
 of every moved byte once), achieved GB/s, L2 atomic requests per unit (claims of the
@@ -17,15 +17,20 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 NCU = "/usr/local/cuda/bin/ncu"
 
 
-def raw(rep):
-    out = subprocess.run([NCU, "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+def sel(skip):
+    """ncu import filter: the skip-th launch of a multi-launch capture (name@skip)."""
+    return ["--launch-skip", str(skip), "--launch-count", "1"] if skip else []
+
+
+def raw(rep, skip=0):
+    out = subprocess.run([NCU, "-i", rep, "--page", "raw", "--csv", *sel(skip)], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     h, u, v = rows[0], rows[1], rows[2]
     return {h[i]: (v[i], u[i]) for i in range(len(h))}
 
 
-def excessive(rep):
-    out = subprocess.run([NCU, "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+def excessive(rep, skip=0):
+    out = subprocess.run([NCU, "-i", rep, "--page", "source", "--csv", "--print-source", "sass", *sel(skip)],
                          capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     h = rows[1]
@@ -63,17 +68,19 @@ def main():
     notes = []
     for spec in specs:
         name, alg, units, desc = spec.split(":", 3)
-        rep = os.path.join(ROOT, "gpurun_out", name + ".ncu-rep")
+        base, _, skip = name.partition("@")   # name@k: the k-th launch of the capture
+        skip = int(skip or 0)
+        rep = os.path.join(ROOT, "gpurun_out", base + ".ncu-rep")
         if not os.path.exists(rep):
             continue
-        d = raw(rep)
+        d = raw(rep, skip)
         t = num(d, "gpu__time_duration.sum")
         rd, wr = num(d, "dram__bytes_read.sum"), num(d, "dram__bytes_write.sum")
         alg, units = float(alg), float(units)
         atom = num(d, "lts__t_requests_op_atom.sum")
         bc = (num(d, "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum") or 0) + \
              (num(d, "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_st.sum") or 0)
-        ex, wtot = excessive(rep)
+        ex, wtot = excessive(rep, skip)
         stalls = []
         for k, (v, _) in d.items():
             if k.startswith("smsp__pcsamp_warps_issue_stalled_") and not k.endswith("not_issued"):

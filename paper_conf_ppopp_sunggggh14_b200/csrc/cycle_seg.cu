@@ -203,7 +203,7 @@ struct SegUaParams {
 };
 
 template <int G, int R>
-__global__ void __launch_bounds__(256, 4) cycle_seg_ua_kernel(const SegUaParams p) {
+__global__ void __launch_bounds__(256, (R >= 5 ? 3 : 4)) cycle_seg_ua_kernel(const SegUaParams p) {
     const uint32_t gl = threadIdx.x % G;
     const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << ((threadIdx.x & 31) - gl));
     const uint64_t w = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) / G;
@@ -376,31 +376,40 @@ struct SegCfg {
 };
 
 // Unaligned units: a walker of G lanes x R vectors covers cap = G*R vectors; a chunk of cw
-// words covers at most (cw + 6) / 4 of them at any phase, so cw + 3 <= 4 cap.  One chunk per
-// unit with the smallest cap (ties: fewest lanes, i.e. most walkers per warp) up to 508
-// words; beyond, greedy 508-word (2032-byte) chunks on 32 x 4 walkers.
+// words covers at most (cw + 6) / 4 of them at any phase, so cw + 3 <= 4 cap.  Units are cut
+// into the fewest equal chunks (multiples of 4 words) that fit the largest walker (32 x 6),
+// and each chunk gets the walker of the smallest cap that holds it (ties: fewest lanes,
+// i.e. most walkers per warp).  R = 3, 5, 6 [r2]: with powers of two only, sizes just above
+// a power-of-two cap (508 B = 33 covering vectors: 16 x 4 = 64 lanes-vectors, half idle)
+// ran ~30 % below their neighbours (IPT_SEG_UA_R2=1 restores the {1, 2, 4} set).
+constexpr int kSegUaRs[] = {1, 2, 3, 4, 5, 6};
 SegCfg seg_cfg_ua(uint64_t S) {
     const uint64_t nw = S / 4;
-    SegCfg c{32, 4, 1, 0, true, 0};
-    uint64_t best = ~0ull;
     const long gmin = env_int("IPT_SEG_UA_G", 8);   // smallest walker width considered
-    for (int G : {8, 16, 32})
-        if (G >= gmin)
-        for (int R = 1; R <= 4; R *= 2) {
-            const uint64_t cap = (uint64_t)G * R;
-            if (nw + 3 <= 4 * cap && cap < best) {
-                best = cap;
-                c.G = G;
-                c.R = R;
-                c.cw = (uint32_t)((nw + 3) & ~3ull);
-            }
-        }
-    if (!c.cw) {
-        c.G = 32;
-        c.R = 4;
+    const bool pow2 = env_int("IPT_SEG_UA_R2", 0) != 0;
+    const int rmax = pow2 ? 4 : 6;
+    const uint64_t maxw = 4ull * 32 * rmax - 3;      // words per chunk on the largest walker
+    SegCfg c{32, rmax, (nw + maxw - 1) / maxw, 0, true, 0};
+    if (pow2 && nw > 508) {   // round-1 rule: greedy 508-word chunks
         c.cw = 508;
         c.nch = (nw + 507) / 508;
+        c.chunk = (uint64_t)c.cw * 4;
+        return c;
     }
+    const uint64_t cw = ((nw + c.nch - 1) / c.nch + 3) & ~3ull;   // balanced, 4-word multiple
+    uint64_t best = ~0ull;
+    for (int G : {8, 16, 32})
+        if (G >= gmin)
+            for (int R : kSegUaRs) {
+                if (R > rmax || (pow2 && (R == 3 || R > 4))) continue;
+                const uint64_t cap = (uint64_t)G * R;
+                if (cw + 3 <= 4 * cap && cap < best) {
+                    best = cap;
+                    c.G = G;
+                    c.R = R;
+                }
+            }
+    c.cw = (uint32_t)cw;
     c.chunk = (uint64_t)c.cw * 4;
     return c;
 }
@@ -443,9 +452,11 @@ void *seg_kernel_ptr() { return (void *)cycle_seg_kernel<G, R>; }
 
 void *seg_kernel(int G, int R, bool ua = false) {
     if (ua) {
-#define IPT_SEG_UA(g, r) if (G == g && R == r) return (void *)cycle_seg_ua_kernel<g, r>;
-        IPT_SEG_UA(8, 1) IPT_SEG_UA(8, 2) IPT_SEG_UA(8, 4) IPT_SEG_UA(16, 1) IPT_SEG_UA(16, 2)
-        IPT_SEG_UA(16, 4) IPT_SEG_UA(32, 1) IPT_SEG_UA(32, 2) IPT_SEG_UA(32, 4)
+#define IPT_SEG_UA(g) if (G == g) switch (R) { \
+        case 1: return (void *)cycle_seg_ua_kernel<g, 1>; case 2: return (void *)cycle_seg_ua_kernel<g, 2>; \
+        case 3: return (void *)cycle_seg_ua_kernel<g, 3>; case 4: return (void *)cycle_seg_ua_kernel<g, 4>; \
+        case 5: return (void *)cycle_seg_ua_kernel<g, 5>; case 6: return (void *)cycle_seg_ua_kernel<g, 6>; }
+        IPT_SEG_UA(8) IPT_SEG_UA(16) IPT_SEG_UA(32)
 #undef IPT_SEG_UA
         return nullptr;
     }

@@ -855,8 +855,10 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
         __syncthreads();
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         // ---- write-out: part A, then part B (chunk by chunk) through the freed shared memory
+        // diag 32 (measurement): stores to a second buffer after the data (out of place)
+        char *const gw = (p.diag & 32) ? g + p.count * p.tile_bytes : g;
         if (ra && !(p.diag & 2))
-            write_out_pan<EB>(p, s0, g, q, divq, p.pstride, r0 / V, ra / V, diva, c0, cvec, NoProbe());
+            write_out_pan<EB>(p, s0, gw, q, divq, p.pstride, r0 / V, ra / V, diva, c0, cvec, NoProbe());
         __syncthreads();
         mark(i, 4);
         if (!CH && nchunk) {   // one chunk: the whole part B through the freed shared memory
@@ -881,7 +883,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
             __syncthreads();
             mark(i, 5);
             if (!(p.diag & 2))
-                write_out_pan<EB>(p, s0, g, q, divq, pstride_b, (r0 + ra) / V, rb / V, divb, c0, cvec, NoProbe());
+                write_out_pan<EB>(p, s0, gw, q, divq, pstride_b, (r0 + ra) / V, rb / V, divb, c0, cvec, NoProbe());
         }
         for (uint32_t k = 0; CH && k < nchunk; ++k) {
             const RfChunk c = rf_chunk(p, k, rb, cvec);
@@ -907,7 +909,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
             }
             __syncthreads();
             if (!(p.diag & 2))
-                write_out_pan<EB>(p, s0, g, q, divq, pstride_b, (r0 + ra + c.r0) / V, c.nr / V,
+                write_out_pan<EB>(p, s0, gw, q, divq, pstride_b, (r0 + ra + c.r0) / V, c.nr / V,
                                   make_fastdiv32_dev(c.nr / V), c0 + c.c0, c.nc, NoProbe());
             __syncthreads();
         }

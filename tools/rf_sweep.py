@@ -16,7 +16,9 @@ if os.environ.get("_CHILD"):
     from inputs import seeded
     res = {}
     for (M, N, eb, cnt) in ast.literal_eval(os.environ["SHAPES"]):
-        t = torch.empty(cnt * M * N, dtype=torch.int32 if eb == 4 else torch.int64, device="cuda")
+        # OOP=1: twice the storage, for IPT_TILE_DIAG=32 (stores to a second buffer after the data)
+        t = torch.empty(cnt * M * N * (2 if os.environ.get("OOP") else 1), dtype=torch.int32 if eb == 4 else torch.int64,
+                        device="cuda")[:cnt * M * N]
         seeded.fill_device_(t, M, N, eb, count=cnt)
         p, q = ipt.plan(M, N, eb, 0, m=M, n=N), ipt.plan(N, M, eb, 0, m=N, n=M)
         kn = ipt.stage_kernels(p, cnt, t)[1]

@@ -388,7 +388,8 @@ SegCfg seg_cfg_ua(uint64_t S) {
     const long gmin = env_int("IPT_SEG_UA_G", 8);   // smallest walker width considered
     const bool pow2 = env_int("IPT_SEG_UA_R2", 0) != 0;
     const int rmax = pow2 ? 4 : 6;
-    const uint64_t maxw = 4ull * 32 * rmax - 3;      // words per chunk on the largest walker
+    // words per chunk on the largest walker: cw + 3 <= 4 cap with cw a multiple of 4
+    const uint64_t maxw = 4ull * 32 * rmax - 4;
     SegCfg c{32, rmax, (nw + maxw - 1) / maxw, 0, true, 0};
     if (pow2 && nw > 508) {   // round-1 rule: greedy 508-word chunks
         c.cw = 508;

@@ -441,6 +441,24 @@ def test_ipt_100_unaligned_realigning_walker(monkeypatch, seg, batch, A, B, s, e
     assert np.array_equal(to_np(t, eb), oracle.permute_inplace(a.copy(), batch, A, B, s))
 
 
+# words per unit at each walker-shape boundary of the segmented unaligned walker (G lanes x R
+# vectors, R = 1..6, the smallest that covers a chunk; 764 words = one full 32 x 6 walker,
+# 765+ two or more balanced chunks), f32 and the f64 equivalents
+UA_WORDS = [5, 29, 61, 93, 127, 157, 189, 253, 317, 381, 509, 764, 765, 766, 1021, 1529, 2301]
+
+
+@pytest.mark.parametrize("s", UA_WORDS)
+def test_ipt_100_unaligned_segmented_walker_shapes(monkeypatch, s):
+    """Every walker shape of cycle_seg_ua (and the chunk split beyond one walker) against
+    the oracle, on a small permutation with long and short cycles."""
+    monkeypatch.setenv("IPT_CYC_SEG", "2")
+    A, B = (13, 7) if s > 700 else (37, 29)
+    a = gen(A * B * s, 4)
+    t = to_dev(a, 4)
+    ipt.ipt_100_(t, 1, A, B, s)
+    assert np.array_equal(to_np(t, 4), oracle.permute_inplace(a.copy(), 1, A, B, s)), s
+
+
 @pytest.mark.parametrize("seg", ["0", "2"])
 @pytest.mark.parametrize("off,batch,A,B,s", [(1, 1, 61, 47, 32), (3, 2, 30, 20, 64), (2, 1, 40, 31, 7)])
 def test_ipt_100_misaligned_base(monkeypatch, seg, off, batch, A, B, s):

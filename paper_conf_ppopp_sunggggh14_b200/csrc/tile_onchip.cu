@@ -130,8 +130,10 @@ __device__ __forceinline__ void write_out(const TileParams &p, uint32_t sbase, c
 }
 
 // As write_out, for a slice held as column panels (tile_group_tma): 16-byte column bjl
-// lives in panel bjl / pw at sbase + panel * pstride, row pitch pw vectors.
-template <int EB, typename Probe>
+// lives in panel bjl / pw at sbase + panel * pstride, row pitch pw vectors.  SWZ: one panel
+// of 128-byte rows in the TMA 128-byte swizzle (vector c of row r at chunk c ^ (r & 7);
+// sbase 1024-byte aligned).
+template <int EB, typename Probe, bool SWZ = false>
 __device__ __forceinline__ void write_out_pan(const TileParams &p, uint32_t sbase, char *g, uint32_t pw,
                                               const FastDiv32 &divpw, uint32_t pstride, uint32_t bi0,
                                               uint32_t mvp, const FastDiv32 &divmvp, uint32_t bj0,
@@ -151,8 +153,8 @@ __device__ __forceinline__ void write_out_pan(const TileParams &p, uint32_t sbas
         E x[V][V];
 #pragma unroll
         for (int kk = 0; kk < V; ++kk) {
-            const uint32_t rho = (uint32_t)((kk + off) % V);
-            const uint4 v = lds128(pb + (bil * V + rho) * pw * 16);
+            const uint32_t rho = (uint32_t)((kk + off) % V), row = bil * V + rho;
+            const uint4 v = SWZ ? lds128(sbase + row * 128 + ((pc ^ (row & 7)) << 4)) : lds128(pb + row * pw * 16);
             unpack<EB>(v, x[kk]);
         }
 #pragma unroll
@@ -715,12 +717,15 @@ __device__ __forceinline__ RfChunk rf_chunk(const TileParams &p, uint32_t k, uin
     return c;
 }
 
-template <int EB, int RV, bool CH>
+template <int EB, int RV, bool CH, bool SWZ = false>
 __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, const __grid_constant__ CUtensorMap tmap) {
     constexpr int V = 16 / EB;
     static_assert(RV % kRfBatch == 0 && RV <= 32, "TMEM holds 32 vectors per thread");
+    static_assert(!(SWZ && CH), "swizzled slices are staged in one chunk");
     extern __shared__ __align__(128) unsigned char smem[];
-    const uint32_t s0 = smem_u32(smem);
+    // SWZ: column slices of exactly 8 vectors (one 128-byte line per row) in the TMA 128-byte
+    // swizzle, whose pattern repeats every 1024 bytes of shared memory address
+    const uint32_t s0 = SWZ ? (smem_u32(smem) + 1023u) & ~1023u : smem_u32(smem);
     const uint32_t K = p.K, rank = blockIdx.x % K, gid = blockIdx.x / K, ng = gridDim.x / K;
     const uint32_t warp = threadIdx.x >> 5, tid = threadIdx.x;
     const uint32_t mv = p.m / V, nvr = p.n / V;
@@ -858,7 +863,7 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
         // diag 32 (measurement): stores to a second buffer after the data (out of place)
         char *const gw = (p.diag & 32) ? g + p.count * p.tile_bytes : g;
         if (ra && !(p.diag & 2))
-            write_out_pan<EB>(p, s0, gw, q, divq, p.pstride, r0 / V, ra / V, diva, c0, cvec, NoProbe());
+            write_out_pan<EB, NoProbe, SWZ>(p, s0, gw, q, divq, p.pstride, r0 / V, ra / V, diva, c0, cvec, NoProbe());
         __syncthreads();
         mark(i, 4);
         if (!CH && nchunk) {   // one chunk: the whole part B through the freed shared memory
@@ -876,14 +881,14 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
                         uint32_t r, c, pn, pc;
                         fdivmod32(e, divc, r, c);
                         fdivmod32(c, divq, pn, pc);
-                        sts128(s0 + pn * pstride_b + (r * q + pc) * 16, v[j]);
+                        sts128(SWZ ? s0 + r * 128 + ((pc ^ (r & 7)) << 4) : s0 + pn * pstride_b + (r * q + pc) * 16, v[j]);
                     }
                 }
             }
             __syncthreads();
             mark(i, 5);
             if (!(p.diag & 2))
-                write_out_pan<EB>(p, s0, gw, q, divq, pstride_b, (r0 + ra) / V, rb / V, divb, c0, cvec, NoProbe());
+                write_out_pan<EB, NoProbe, SWZ>(p, s0, gw, q, divq, pstride_b, (r0 + ra) / V, rb / V, divb, c0, cvec, NoProbe());
         }
         for (uint32_t k = 0; CH && k < nchunk; ++k) {
             const RfChunk c = rf_chunk(p, k, rb, cvec);
@@ -1786,6 +1791,7 @@ cudaError_t launch_group_db(const StageDesc &d, TileParams p, const GroupCfg &g,
 struct RfCfg {
     int K = 0, rv = 0;
     bool colsplit = false;
+    bool swz = false;      // column slices of one 128-byte line per row, TMA 128-byte swizzle
     uint32_t q = 0, npan = 0, rows_a = 0, rows_b = 0, cpan = 0, box_rows = 0, ralign = 0;
     size_t pstride = 0, smem = 0;
 };
@@ -1869,6 +1875,45 @@ static RfCfg rf_search(int64_t A, int64_t B, int eb, int device, bool cs, bool c
     return c;
 }
 
+// Column slices of exactly one 128-byte line per row (8 vectors): K = B*eb/128 CTAs, which
+// must be at least 3/4 of the SMs (the rest idle).  Part A lands by TMA in the 128-byte
+// swizzle (conflict-free write-out reads at pitch 128 B), part B is restaged through the
+// same region in one chunk.  Every CTA's pieces of the input rows are whole lines -- no
+// sector is shared between two CTAs.
+static RfCfg rf_search_swz(int64_t A, int64_t B, int eb, int device) {
+    RfCfg c;
+    const DevProps dp = dev_props(device);
+    const int V = 16 / eb;
+    const int64_t nvr = B / V;
+    if (nvr % 8) return c;
+    const int64_t K = nvr / 8;
+    if (K > dp.sms || 4 * K < 3 * (int64_t)dp.sms) return c;
+    const long budget = env_int("IPT_TILE_SMEM_MAX", dp.smem_optin) - 2048;   // + 1 KB alignment slack
+    for (int64_t ra = std::min<int64_t>(A, budget / 128) / 8 * 8; ra >= 8; ra -= 8) {
+        uint32_t br = 0;
+        for (uint32_t b = 256; b >= 8; b -= 8)
+            if (ra % b == 0) { br = b; break; }
+        if (!br) continue;
+        const int64_t rb = A - ra;
+        if (rb * 8 > (int64_t)kRfThreads * kRfMaxRV || rb * 128 > budget) return c;   // smaller A: more B
+        c.K = (int)K;
+        c.colsplit = true;
+        c.swz = true;
+        c.ralign = 8;
+        c.q = 8;
+        c.npan = 1;
+        c.rows_a = (uint32_t)ra;
+        c.rows_b = (uint32_t)std::max<int64_t>(rb, V);
+        c.cpan = 1;
+        c.box_rows = br;
+        c.rv = (int)((rb * 8 + kRfThreads - 1) / kRfThreads);
+        c.pstride = (size_t)ra * 128;
+        c.smem = 1024 + (size_t)std::max(ra, rb) * 128;
+        return c;
+    }
+    return c;
+}
+
 static RfCfg rf_cfg(int64_t A, int64_t B, int eb, int device) {
     if ((eb != 4 && eb != 8) || !vec_ok(A, B, eb) || !env_int("IPT_TILE_RF", 1)) return RfCfg{};
     static std::mutex mu;
@@ -1896,6 +1941,7 @@ static RfCfg rf_cfg(int64_t A, int64_t B, int eb, int device) {
     const int64_t ral = rab > 16 ? rab / 16 : 1;   // V-blocks are 16 bytes of an output row
     RfCfg c;
     const long fcs = env_int("IPT_TILE_RF_CS", -1);   // measurement: force the split direction
+    if (!row_first && fcs != 0 && env_int("IPT_TILE_RF_SWZ", 1)) c = rf_search_swz(A, B, eb, device);
     for (int pass = 0; pass < 4 && !c.K; ++pass) {
         const bool cs = (pass & 1) ? row_first : !row_first;
         if (fcs >= 0 && cs != (fcs != 0)) continue;
@@ -1927,7 +1973,8 @@ cudaError_t launch_group_rf(const StageDesc &d, TileParams p, const RfCfg &c, vo
         cuuint32_t box[2] = {c.q * (uint32_t)V, c.box_rows};
         cuuint32_t estr[2] = {1, 1};
         r = enc(&tm, EB == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 2, d.base,
-                dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                c.swz ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
                 CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
         p.rres = 0;
     } else {        // strided batch of single tiles: (columns, rows, tiles), tile stride ostride
@@ -1937,7 +1984,8 @@ cudaError_t launch_group_rf(const StageDesc &d, TileParams p, const RfCfg &c, vo
         cuuint32_t box[3] = {c.q * (uint32_t)V, c.box_rows, 1};
         cuuint32_t estr[3] = {1, 1, 1};
         r = enc(&tm, EB == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 3, d.base,
-                dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                c.swz ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
                 CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
         p.rres = 1;
     }
@@ -1975,7 +2023,8 @@ cudaError_t launch_group_rf(const StageDesc &d, TileParams p, const RfCfg &c, vo
         : std::max((mvv / ral + c.K - 1) / c.K * ral, mvv - (mvv / ral) * (c.K - 1) / c.K * ral) * V;
     const int64_t rbm = rmax - (int64_t)c.rows_a;   // max rows in TMEM
     const bool ch = rbm > (int64_t)c.rows_b || c.cpan < c.npan;
-#define IPT_RF(R) if (rv == R) kern = ch ? (const void *)tile_group_rf<EB, R, true> : (const void *)tile_group_rf<EB, R, false>;
+#define IPT_RF(R) if (!kern && rv == R) kern = c.swz ? (ch ? nullptr : (const void *)tile_group_rf<EB, R, false, true>) \
+        : ch ? (const void *)tile_group_rf<EB, R, true> : (const void *)tile_group_rf<EB, R, false>;
     IPT_RF(8) IPT_RF(16) IPT_RF(24) IPT_RF(32)
 #undef IPT_RF
     if (!kern) return cudaErrorNotSupported;

@@ -230,6 +230,10 @@ RF_CASES = [  # (M, N, eb, count, stride pad in elements, smem budget override o
     (720, 1800, 4, 2, 0, 60000),       # everything in shared memory (no TMEM part)
     (4096, 3000, 4, 2, 0, -16),        # row slices on any 16-byte boundary (IPT_TILE_RF_RALIGN=0)
     (4000, 3200, 4, 2, 0, -64),        # 64-byte aligned row slices
+    (600, 4096, 4, 3, 0, 0),           # column slices of one 128-byte line, TMA 128-byte swizzle:
+    (2500, 4096, 4, 1, 0, 0),          #   no TMEM part / a TMEM part restaged swizzled,
+    (1500, 2048, 8, 2, 24, 0),         #   float64, strided (3-D map)
+    (3000, 4096, 4, 2, 0, -1),         # the same tile with the swizzled slices off (-1)
 ]
 
 
@@ -242,6 +246,8 @@ def test_tile_group_rf(monkeypatch, M, N, eb, count, pad, smem):
     monkeypatch.setenv("IPT_TILE_RF_FORCE", "1")
     if smem > 0:
         monkeypatch.setenv("IPT_TILE_SMEM_MAX", str(smem))
+    elif smem == -1:
+        monkeypatch.setenv("IPT_TILE_RF_SWZ", "0")
     elif smem < 0:
         monkeypatch.setenv("IPT_TILE_RF_RALIGN", str(-smem if smem != -16 else 0))
     dt = torch.int32 if eb == 4 else torch.int64

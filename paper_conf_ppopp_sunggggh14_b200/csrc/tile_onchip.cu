@@ -696,6 +696,10 @@ __device__ __forceinline__ uint4 tm_ld4(uint32_t taddr) {
 }
 
 constexpr int kRfBatch = 8;   // part-B vectors per thread in registers at a time
+// Part-B loads in flight per thread on the one-chunk path: half of the thread's vectors
+// (two round trips), at least 8 -- rv = 24: 12 per batch, measured C5 4.92 -> 5.01 TB/s
+// (8: 4.92, 10: 4.89, 12: 5.01, 14: 4.93, 16: 4.88, 24: 4.92; 512 matrices)
+constexpr int rf_load_batch(int rv) { return rv / 2 < 8 ? 8 : rv / 2; }
 
 // Part B is handled in chunks (cb rows x cpan panels of the slice, staged through a
 // region of shared memory after part A's): chunk k's vectors are numbered consecutively
@@ -804,26 +808,28 @@ __global__ void __launch_bounds__(512, 1) tile_group_rf(const TileParams p, cons
         // ---- part B: 16-byte loads parked in TMEM (thread E % 512 holds vector E in its
         // columns 4 * (E / 512); with several chunks, chunk k's vectors start at base_k)
         if (!(p.diag & 4) && !CH) {   // one chunk: every thread's vectors E < nvb
-            // (batches of kRfBatch loads, each parked before the next is issued: measured
-            // faster than 2 batches or all of a thread's loads in flight -- 4.39 vs 4.34 TB/s
-            // on C5, 3.3 vs 3.0 on one C1 matrix)
+            // (batches of LB loads, each parked before the next is issued: all of a thread's
+            // loads in flight measured slower -- 4.39 vs 4.34 TB/s on C5, 3.3 vs 3.0 on one
+            // C1 matrix, first version)
             const char *gb = g + ((size_t)(r0 + ra) * nvr + c0) * 16;
 #pragma unroll 1
-            for (int u0 = 0; u0 < RV; u0 += kRfBatch) {
+            constexpr int LB = rf_load_batch(RV);
+            for (int u0 = 0; u0 < RV; u0 += LB) {
                 if ((uint32_t)u0 * 512 >= nvb) break;
-                uint4 v[kRfBatch];
+                uint4 v[LB];
 #pragma unroll
-                for (int j = 0; j < kRfBatch; ++j) {
+                for (int j = 0; j < LB; ++j) {
                     const uint32_t e = tid + (uint32_t)(u0 + j) * 512;
                     v[j] = make_uint4(0, 0, 0, 0);
-                    if (e < nvb) {
+                    if (u0 + j < RV && e < nvb) {
                         uint32_t r, c;
                         fdivmod32(e, divc, r, c);
                         v[j] = ld_cg<16>(gb + ((size_t)r * nvr + c) * 16);
                     }
                 }
 #pragma unroll
-                for (int j = 0; j < kRfBatch; ++j) tm_st4(taddr + 4u * (uint32_t)(u0 + j), v[j]);
+                for (int j = 0; j < LB; ++j)
+                    if (u0 + j < RV) tm_st4(taddr + 4u * (uint32_t)(u0 + j), v[j]);
             }
             asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
             mark(i, 1);

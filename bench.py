@@ -11,9 +11,13 @@ peak scaled by the number S of non-identity stages executed.
 Headline (N = 1 and every N): the largest single-GPU BASELINE config, configs[4] = C5, a
 batch of 512 independent 4096 x 3000 float32 matrices (25.17 GB), partitioned across the
 N ranks by partition.BatchShard (contiguous blocks, no collective on the data path,
-P:240).  One step = one ipt_transpose_batched call per rank over its shard (the
-orientation alternates step to step: 4096 x 3000 -> 3000 x 4096 -> ...).  Inputs exceed
-the 126 MB L2, so no flush is needed.
+P:240).  One step = one ipt_transpose_batched call per rank over its shard: every
+matrix, 4096 x 3000, becomes its 3000 x 4096 transpose; the next step reads the same
+storage as the next 4096 x 3000 matrices (`--orientation fixed`, default: the configured
+shape every step; `alternate` transposes back and forth, 4096 x 3000 and 3000 x 4096 on
+alternate steps).  Two extra untimed steps of the reverse shape are reported for context
+(`per_shape_reverse`).  The final state is checked on samples against the composition of
+every transposition applied since the fill.  Inputs exceed the 126 MB L2: no flush.
 
 Sub-records (N = 1, rank 0, after the headline's timed region; `--sub`): every other
 BASELINE config, each matrix timed on its own with per-step CUDA events -- C1 (cold L2),
@@ -302,19 +306,26 @@ def emit(line, args):
 
 
 # ---------------------------------------------------------------------- ours: common
-def _verify(t, M, N, eb, transposed, t0=0, count=1, nsamp=4096, seed=0):
-    """Sampled definition check of `count` packed matrices (generator index t0 + k):
-    after a transpose, position p = j*M + i holds v(i*N + j)."""
+def _verify(t, M, N, eb, transposed, t0=0, count=1, nsamp=4096, seed=0, seq=None):
+    """Sampled definition check of `count` packed matrices (generator index t0 + k).
+    One a x b transpose moves position p = i*b + j to j*a + i; `seq` lists the (a, b)
+    transposes applied since the fill, in order (default: one M x N transpose if
+    `transposed`, none otherwise), and a sampled position's source is found by undoing
+    them in reverse order."""
     import torch
     from inputs import seeded
 
     n = M * N
+    if seq is None:
+        seq = [(M, N)] if transposed else []
     g = torch.Generator(device="cpu").manual_seed(seed)
     ok = True
     for k in sorted({0, count // 2, count - 1}):
         pos = torch.randint(0, n, (nsamp,), generator=g).to(t.device)
         seg = t[k * n:(k + 1) * n]
-        src = (pos % M) * N + pos // M if transposed else pos
+        src = pos.clone()
+        for (a, b) in reversed(seq):   # position d = j*a + i came from i*b + j
+            src = (src % a) * b + src // a
         exp = seeded.values_torch_sample(src + (t0 + k) * n, eb)
         ok &= bool(torch.equal(seg[pos], exp.to(seg.dtype)))
     return ok
@@ -477,6 +488,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--orientation", default="fixed", choices=["fixed", "alternate"],
+                    help="headline steps: the configured M x N every step (fixed) or M x N and "
+                         "N x M on alternate steps")
     ap.add_argument("--record", default=os.environ.get("IPT_BENCH_RECORD"),
                     help="also append the JSON line, with a UTC timestamp and the git revision, "
                          "to this JSONL run-record file")
@@ -548,15 +562,21 @@ def main():
             ipt.transpose_batched_(t, cnt, a, b, plan_=plans[(a, b)])   # back to M x N
     torch.cuda.synchronize()
     orient = [False] * len(mats)
+    seqs = [[] for _ in mats]   # transposes applied since the fill (the setup above is net identity)
+    fixed = args.orientation == "fixed"
 
-    def one_step(evs=None):
+    def one_step(evs=None, reverse=False):
         for i, (t, M, N, cnt, _) in enumerate(mats):
             if cnt == 0:
                 continue
-            a, b = (N, M) if orient[i] else (M, N)
+            if fixed:
+                a, b = (N, M) if reverse else (M, N)
+            else:
+                a, b = (N, M) if orient[i] else (M, N)
+                orient[i] = not orient[i]
             ipt.transpose_batched_(t, cnt, a, b, plan_=plans[(a, b)],
                                    events=evs[i] if evs is not None else None)
-            orient[i] = not orient[i]
+            seqs[i].append((a, b))
 
     for _ in range(args.warmup):
         one_step()
@@ -631,7 +651,7 @@ def main():
         for i, (t, M, N, cnt, _) in enumerate(mats):
             if cnt == 0:
                 continue
-            a, b = (N, M) if orient_sim[i] else (M, N)
+            a, b = (M, N) if fixed else ((N, M) if orient_sim[i] else (M, N))
             p = plans[(a, b)]
             S_bytes += 2 * a * b * eb * cnt * p.n_stages
             if timed:
@@ -667,15 +687,30 @@ def main():
                     "peak_source": peak_src, "launches": kn, "avg_launch_ms": round(kms / kn, 4),
                     "share_of_step": round(kms / ev_ms, 4) if ev_ms else None,
                     "algorithmic_bytes_per_launch": kb // kn,
-                    "stage_events": f"last {n_ev} of {args.steps} timed steps (both orientations)",
+                    "stage_events": f"last {n_ev} of {args.steps} timed steps" + ("" if fixed else " (both orientations)"),
                     "per_kernel": {k: {"ms": round(v[0], 3), "gbs": round(v[1] / (v[0] / 1e3) / 1e9, 1),
                                        "launches": v[2]} for k, v in kern.items()}}
+
+    # ---- the reverse shape (N x M) for context: two untimed steps with stage events
+    per_shape_rev = {}
+    if fixed and sh is not None and sh.count:
+        for _ in range(2):
+            ev_r = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in mats]
+            one_step(ev_r, reverse=True)
+            torch.cuda.synchronize()
+            for i, (t, M, N, cnt, _) in enumerate(mats):
+                ms = [ev_r[i][st].elapsed_time(ev_r[i][st + 1]) for st in range(3)]
+                p = plans[(N, M)]
+                per_shape_rev[f"{N}x{M}"] = {"count": cnt, "m": p.m, "n": p.n, "S": p.n_stages,
+                                             "eff_gbs": round(2 * M * N * eb * cnt / (sum(ms) / 1e3) / 1e9, 1),
+                                             "stages": _stage_rec(ipt, p, cnt, t, N, M, eb, ms),
+                                             "note": "untimed, not in value: the reverse shape for context"}
 
     # ---- verification of the final state (sampled definition check, every rank)
     ok = True
     for i, (t, M, N, cnt, t0) in enumerate(mats):
         if cnt:
-            ok &= _verify(t, M, N, eb, orient[i], t0=t0, count=cnt, seed=i)
+            ok &= _verify(t, M, N, eb, False, t0=t0, count=cnt, seed=i, seq=seqs[i])
     ok = part.all_ok(ok, red_dev)
     for m in mats:
         m[0] = None
@@ -724,9 +759,14 @@ def main():
                        "parallelism": (f"batch shards x{world} (no collective on the data path)"
                                        if sh is not None else f"replicas x{world}"),
                        "planning": (f"ipt_plan_autotune, {args.autotune} candidates per shape "
-                                    "(before the timed region)") if args.autotune > 1 else "cost model"},
+                                    "(before the timed region)") if args.autotune > 1 else "cost model",
+                       "orientation": ("fixed: every step transposes the configured shape (the previous "
+                                       "step's transposes re-read as the next inputs; final state checked "
+                                       "against the composition of all transposes)" if fixed else
+                                       "alternate: the configured shape and its transpose on alternate steps")},
             "hbm_frac_stage_scaled": round(stage_scaled, 4),
-            "per_shape": per_shape, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "per_shape": per_shape, "per_shape_reverse": per_shape_rev or None,
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches, "clocks": clk, "verified": ok, "sub": subs,
         }
         emit(line, args)

@@ -129,3 +129,26 @@ def test_workloads_lists():
         assert s in W.SWEEP_ALL
     assert len(set(W.SWEEP_ALL)) == len(W.SWEEP_ALL)
     assert (9797, 13081) in W.SWEEP_ALL and (10007, 19997) in W.PRIMES
+
+
+def test_bench_verify_composed_transposes():
+    """bench._verify undoes a sequence of transposes (the fixed-orientation headline: the
+    M x N result re-read as the next M x N input, plus N x M steps): checked against
+    numpy transposes of the generator values on CPU tensors, and a wrong sequence fails."""
+    import importlib.util
+    import torch
+
+    spec = importlib.util.spec_from_file_location("bench_mod", os.path.join(ROOT, "bench.py"))
+    bench = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(bench)
+    for eb in (4, 8):
+        count, M, N, t0 = 3, 6, 10, 5
+        x = seeded.values_np(np.arange(t0 * M * N, (t0 + count) * M * N, dtype=np.uint64), eb)
+        x = x.reshape(count, M * N)
+        seq = [(M, N), (M, N), (N, M), (M, N), (M, N)]
+        for (a, b) in seq:
+            x = np.ascontiguousarray(x.reshape(count, a, b).transpose(0, 2, 1)).reshape(count, M * N)
+        dt = torch.int32 if eb == 4 else torch.int64
+        t = torch.from_numpy(x.reshape(-1).view(np.int32 if eb == 4 else np.int64).copy()).to(dt)
+        assert bench._verify(t, M, N, eb, False, t0=t0, count=count, nsamp=256, seq=seq)
+        assert not bench._verify(t, M, N, eb, False, t0=t0, count=count, nsamp=256, seq=seq[:-1])

@@ -24,14 +24,17 @@ def main(timed=5):
         d = L.setdefault(int(r[ci["ID"]]), {"name": r[ci["Kernel Name"]]})
         d[r[ci["Metric Name"]]] = float(r[ci["Metric Value"]].replace(",", "")) * SCALE.get(r[ci["Metric Unit"]], 1)
     ipt_l = [(k, v) for k, v in L.items() if "ipt::" in v["name"]]
+    rev = ipt_l[-2:]              # the two untimed reverse-shape steps after the timed region
+    ipt_l = ipt_l[:-2]
     last = ipt_l[-timed:]
     alg = 2 * 512 * 4096 * 3000 * 4 / 1e9
     out = ["# r02: ncu launch list of `python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu --sub none` (C5 headline)", "",
            "Cold-cache, serialised (`--clock-control none`); the shares and per-launch DRAM bytes are what count, not",
            "absolute times. Earlier libipt launches in the list are the autotune candidates (`ipt_plan_autotune_batched`,",
            "8 candidates per orientation: 1-stage whole-GPU tiles vs 2-stage panel plans), all before the timed region.",
-           f"The {timed} launches below are the 3 warm-up + 2 timed steps; the orientation alternates (4096x3000:",
-           "row-split slices, `tile_group_rf<4, 24, 0>`; 3000x4096: column-split slices, `<4, 16, 0>`).", "",
+           f"The {timed} launches below are the 3 warm-up + 2 timed steps, every one a 4096x3000 -> 3000x4096",
+           "transposition of the 512 matrices (row-split slices); the bench's two untimed reverse-shape steps",
+           "(3000x4096, swizzled column slices) follow the table.", "",
            "| launch | kernel | µs | DRAM read GB | DRAM write GB | algorithmic GB (read+write) | DRAM / algorithmic |",
            "|---|---|---|---|---|---|---|"]
     tb = tt = 0.0
@@ -40,6 +43,10 @@ def main(timed=5):
         tb += (rd + wr) * 1e9
         tt += t
         out.append(f"| {k} | `{v['name'][:60]}` | {t:.1f} | {rd:.3f} | {wr:.3f} | {alg:.3f} | {(rd + wr) / alg:.4f} |")
+    for k, v in rev:
+        rd, wr, t = v["dram__bytes_read.sum"] / 1e9, v["dram__bytes_write.sum"] / 1e9, v["gpu__time_duration.sum"]
+        out.append(f"| {k} (reverse, untimed) | `{v['name'][:60]}` | {t:.1f} | {rd:.3f} | {wr:.3f} | {alg:.3f} | "
+                   f"{(rd + wr) / alg:.4f} |")
     out += ["", f"tile_group_rf is 100 % of the timed step (one launch per step, 512 matrices). Per launch: "
             f"{tb / timed / 1e9:.3f} GB of DRAM traffic for {alg:.3f} GB algorithmic; average {tt / timed:.0f} µs "
             f"under ncu ({alg * 1e6 / (tt / timed):.0f} GB/s)."]

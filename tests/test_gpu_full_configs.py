@@ -107,6 +107,47 @@ def test_c5_full_batch_one_gpu():
     torch.cuda.empty_cache()
 
 
+def test_c5_fixed_orientation_steps():
+    """The bench's headline steps (--orientation fixed): the full 512-matrix C5 batch
+    transposed as 4096 x 3000 three times in a row (each result re-read as the next
+    4096 x 3000 input), then once as 3000 x 4096 -- every element of three matrices and the
+    first element block of all 512 checked against the composed definition (each a x b
+    transpose moves position i*b + j to j*a + i)."""
+    count, (M, N) = W.C5_COUNT, W.C5_SHAPE
+    free, _ = torch.cuda.mem_get_info()
+    if free < count * M * N * 4 + (6 << 30):
+        pytest.skip("needs ~32 GB of free device memory")
+    n = M * N
+    t = torch.empty(count * n, dtype=torch.int32, device="cuda")
+    seeded.fill_device_(t, M, N, 4, count=count)
+    p = ipt.plan_autotune_batched(t, count, M, N, AUTOTUNE)
+    q = ipt.plan_autotune_batched(t, count, N, M, AUTOTUNE)
+    seq = [(M, N)] * 3 + [(N, M)]
+    for (a, b) in seq:
+        ipt.transpose_batched_(t, count, a, b, plan_=p if (a, b) == (M, N) else q)
+    torch.cuda.synchronize()
+
+    def src_of(pos):
+        for (a, b) in reversed(seq):
+            pos = (pos % a) * b + pos // a
+        return pos
+
+    CH = 1 << 26
+    for k in (0, count // 2, count - 1):         # every element of three matrices
+        flat = t[k * n:(k + 1) * n]
+        for p0 in range(0, n, CH):
+            pos = torch.arange(p0, min(n, p0 + CH), device="cuda", dtype=torch.int64)
+            exp = seeded.values_torch_sample(src_of(pos) + k * n, 4)
+            assert torch.equal(flat[p0:p0 + pos.numel()], exp.to(torch.int32)), k
+    pos = torch.arange(0, 4096, device="cuda", dtype=torch.int64)
+    src = src_of(pos)
+    for k in range(count):                       # a block of every matrix
+        exp = seeded.values_torch_sample(src + k * n, 4)
+        assert torch.equal(t[k * n:k * n + 4096], exp.to(torch.int32)), k
+    del t
+    torch.cuda.empty_cache()
+
+
 # ------------------------------------------------------- capture-safety (ADVICE r1)
 def _mat(M, N, t0=0):
     t = torch.empty(M * N, dtype=torch.int32, device="cuda")

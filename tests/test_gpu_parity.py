@@ -1159,3 +1159,21 @@ def test_cuda_graph_batched():
         blk = src[k * stride:k * stride + M * N].copy()
         assert np.array_equal(got[k * stride:k * stride + M * N], oracle.transpose_inplace(blk, M, N)), k
         assert np.array_equal(got[k * stride + M * N:(k + 1) * stride], src[k * stride + M * N:(k + 1) * stride])
+
+
+@pytest.mark.parametrize("eb", [1, 2, 4, 8, 16])
+def test_public_api_degenerate_shapes(eb):
+    """The planner path of ipt_transpose / ipt_transpose_batched on the degenerate cases:
+    1 x N and M x 1 (no-ops, C6), 1 x 1, 2 x 2, 2 x 3, a prime x prime pair, an empty batch
+    (count 0: nothing touched) and a batch of one -- each against the oracle."""
+    for (M, N) in [(1, 17), (23, 1), (1, 1), (2, 2), (2, 3), (13, 7), (3, 1024)]:
+        a = gen(M * N, eb)
+        t = to_dev(a, eb)
+        ipt.transpose_(t, M, N, elem_bytes=eb)
+        assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), 1, M, N, 1, eb)), (M, N, eb)
+    a = gen(64, eb)
+    t = to_dev(a, eb)
+    ipt.transpose_batched_(t, 0, 4, 16, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), a)
+    ipt.transpose_batched_(t, 1, 4, 16, elem_bytes=eb)
+    assert np.array_equal(to_np(t, eb), oracle_P(a.copy(), 1, 4, 16, 1, eb))

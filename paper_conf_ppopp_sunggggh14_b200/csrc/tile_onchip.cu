@@ -148,12 +148,15 @@ __device__ __forceinline__ void write_out_pan(const TileParams &p, uint32_t sbas
         fdivmod32(blk, divmvp, bjl, bil);
         fdivmod32(bjl, divpw, pan, pc);
         const uint32_t bi = bi0 + bil, bj = bj0 + bjl;
-        // lane rotation of the V rows a thread reads (undone by rotate_sel): conflict-free
-        // LDS.128 for >= 8 consecutive V-row blocks; for V = 4 the offset 2(bil/2) + bil/4
-        // also brings slices of 4 blocks (the rf row slices' part A) from 1.31 to 1.06
-        // wavefronts per access (bank model over all quarter-warp alignments and odd
-        // pitches; 3-7 blocks 1.21-1.35 either way).  rf 4096x3000: 5.11 -> 5.19 TB/s
-        const int off = V == 4 ? (int)((((bil >> 1) << 1) + (bil >> 2)) & 3) : (int)((bil / ROT) % V);
+        // lane rotation of the V rows a thread reads (undone by rotate_sel): (bil / ROT) mod V
+        // is conflict-free for runs of >= 8 consecutive V-row blocks at any quarter-warp
+        // alignment; for V = 4 and mvp = 4 mod 8 blocks per column (the rf row slices' part A
+        // of 4 blocks), 2(bil/2) + bil/4 takes 1.31-1.5 wavefronts per access to 1.0 (bank
+        // model over all quarter-warp alignments, odd pitches and the 128-byte swizzle;
+        // it is worse for other block counts, e.g. 450: 1.17 vs 1.01).  rf 4096x3000:
+        // 5.11 -> 5.19 TB/s
+        const int off = (V == 4 && (mvp & 7) == 4) ? (int)((((bil >> 1) << 1) + (bil >> 2)) & 3)
+                                                   : (int)((bil / ROT) % V);
         const uint32_t pb = sbase + pan * pstride + pc * 16;
         E x[V][V];
 #pragma unroll

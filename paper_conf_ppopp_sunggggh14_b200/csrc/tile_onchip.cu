@@ -1079,16 +1079,21 @@ __global__ void __launch_bounds__(512, 1) tile_group_generic(const TileParams p)
             const uint32_t srow = sb + i * Q * 16;
             const uint32_t cfirst = ch * CH * PV;
             char *out = g + ((uint64_t)(c0 + cfirst) * p.m + r0 + i) * EB;
+            // the phase o is the row's (c is a multiple of PV): consecutive column blocks
+            // share a vector -- carried instead of loaded twice
+            const uint32_t o = sh % PV, v0 = (sh + cfirst) / PV;
+            uint4 cur = lds128(srow + v0 * 16);
 #pragma unroll 2
             for (uint32_t cbl = 0; cbl < CH; ++cbl) {
                 const uint32_t c = cfirst + cbl * PV;
                 if (c >= L) break;
-                const uint32_t w = sh + c, v = w / PV, o = w % PV;
+                const uint4 nxt = lds128(srow + (v0 + cbl + 1) * 16);
                 E x[2 * PV];
                 {
                     E ex[PV], ey[PV];
-                    unpack<EB>(lds128(srow + v * 16), ex);
-                    unpack<EB>(lds128(srow + (v + 1) * 16), ey);
+                    unpack<EB>(cur, ex);
+                    unpack<EB>(nxt, ey);
+                    cur = nxt;
 #pragma unroll
                     for (uint32_t k = 0; k < PV; ++k) { x[k] = ex[k]; x[PV + k] = ey[k]; }
                 }

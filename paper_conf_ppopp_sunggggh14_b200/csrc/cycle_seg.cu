@@ -156,21 +156,18 @@ __global__ void __launch_bounds__(256, 4) cycle_seg_kernel(const SegParams p) {
 template <int G, int R>
 __device__ __forceinline__ uint4 group_vec_nb(const uint4 (&a)[R], int r, uint32_t gl, int dir, unsigned gmask) {
     const int src = ((int)gl + dir + G) % G;
-    const bool wrap = (int)gl + dir < 0 || (int)gl + dir >= G;
-    // the neighbouring register (compile-time indices: no local-memory array)
+    // the neighbouring register (compile-time indices: no local-memory array).  Lane s's
+    // only receiver is lane s - dir; the receiver that wraps around the group (lane G-1
+    // for dir = +1, lane 0 for dir = -1) wants the sender's neighbouring register, so the
+    // edge sender (lane 0, resp. G-1) sends that one instead: one shuffle per word.
     const uint4 o = dir > 0 ? a[r + 1 < R ? r + 1 : R - 1] : a[r > 0 ? r - 1 : 0];
-    uint4 x, y;
-    x.x = __shfl_sync(gmask, a[r].x, src, G);
-    x.y = __shfl_sync(gmask, a[r].y, src, G);
-    x.z = __shfl_sync(gmask, a[r].z, src, G);
-    x.w = __shfl_sync(gmask, a[r].w, src, G);
-    if (R > 1) {
-        y.x = __shfl_sync(gmask, o.x, src, G);
-        y.y = __shfl_sync(gmask, o.y, src, G);
-        y.z = __shfl_sync(gmask, o.z, src, G);
-        y.w = __shfl_sync(gmask, o.w, src, G);
-        if (wrap) x = y;
-    }
+    const bool edge = R > 1 && (dir > 0 ? gl == 0 : gl == G - 1);
+    const uint4 snd = edge ? o : a[r];
+    uint4 x;
+    x.x = __shfl_sync(gmask, snd.x, src, G);
+    x.y = __shfl_sync(gmask, snd.y, src, G);
+    x.z = __shfl_sync(gmask, snd.z, src, G);
+    x.w = __shfl_sync(gmask, snd.w, src, G);
     return x;
 }
 __device__ __forceinline__ uint32_t w4(const uint4 &v, int k) {

@@ -28,10 +28,11 @@ def main(timed=5):
     ipt_l = ipt_l[:-2]
     last = ipt_l[-timed:]
     alg = 2 * 512 * 4096 * 3000 * 4 / 1e9
-    out = ["# r02: ncu launch list of `python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu --sub none` (C5 headline)", "",
+    out = ["# r02: ncu launch list of `python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu --sub none --autotune 1` (C5 headline)", "",
            "Cold-cache, serialised (`--clock-control none`); the shares and per-launch DRAM bytes are what count, not",
-           "absolute times. Earlier libipt launches in the list are the autotune candidates (`ipt_plan_autotune_batched`,",
-           "8 candidates per orientation: 1-stage whole-GPU tiles vs 2-stage panel plans), all before the timed region.",
+           "absolute times. `--autotune 1` (the cost model's plan, the same plan the timed bench run's autotune picks:",
+           "`config.plans` of `profiles/r02_bench.json`): under ncu's serialised replay the autotune timings are",
+           "distorted (one capture picked a 2-stage plan). Earlier libipt launches are the plan-setup transposes.",
            f"The {timed} launches below are the 3 warm-up + 2 timed steps, every one a 4096x3000 -> 3000x4096",
            "transposition of the 512 matrices (row-split slices); the bench's two untimed reverse-shape steps",
            "(3000x4096, swizzled column slices) follow the table.", "",
@@ -53,7 +54,7 @@ def main(timed=5):
     c = collections.defaultdict(list)
     for k, v in ipt_l[:-timed]:
         c[v["name"].split("(")[0].replace("void ipt::", "")].append(v["gpu__time_duration.sum"])
-    out += ["", "Autotune candidates seen (µs per launch, 512 matrices): " +
+    out += ["", "Other libipt launches before the timed region (µs per launch, 512 matrices): " +
             "; ".join(f"`{n}` {min(t):.0f}–{max(t):.0f}" for n, t in c.items())]
     open(os.path.join(ROOT, "profiles", "r02_launches_c5.md"), "w").write("\n".join(out) + "\n")
     tj = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))

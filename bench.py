@@ -582,7 +582,7 @@ def main():
         one_step()
     torch.cuda.synchronize()
 
-    # per-stage events on the last two timed steps (both orientations), created up front
+    # per-stage events on the last two timed steps, created up front
     n_ev = 2
     evs = [[[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in mats]
            for _ in range(n_ev)]
